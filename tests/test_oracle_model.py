@@ -1,0 +1,189 @@
+"""Pins of the model oracle (oracle/model_oracle.py) and of the hexagon
+geometry readings, against hand arithmetic from the paper's own constants,
+the paper's special cases, a brute-force enumeration of the tiling, and
+invariants.  PAPER.md §4 (Eqs. 2-30), §5 Tables 2-4, §6.1 (Eq. 31)."""
+import math
+import random
+
+import pytest
+
+from oracle import hex_geometry as hg
+from oracle import model_oracle as mo
+
+
+def test_hand_worked_gradient2d_gtx980():
+    """Re-derived by hand from Tables 2-4 for the Fig. 5 problem
+    (Gradient-2D, S1 = S2 = T = 8192) at tile
+    (tT, tS1, tS2) = (8, 8, 256), literal equations:
+      Nw = 2*1024 + 1 = 2049          (Eq. 3, T mod tT = 0 -> eps = 1)
+      wtile = 14                       (Eq. 4)
+      w = ceil(8192/24) = 342          (Eq. 5)
+      Mtile = 2*17*265 = 9010 words = 36040 B <= 48 KB      (Eq. 19)
+      k = min(32, floor(98304/36040)) = 2                   (Eq. 11/31)
+      mi = mo = 256*(8+16) = 6144      (Eq. 13)
+      L = 7.36e-3 s/GB * 4e-9 = 2.944e-11 s/word
+      m' = 12288*2.944e-11 + 2*7.96e-10 = 3.63355e-7 s       (Eq. 14)
+      c = 2*6.09e-8*(16+20+24+28) + 8*7.96e-10 = 1.0724768e-5 s  (Eq. 15)
+      N2 = ceil(8200/256) = 33
+      Tprism = m' + 2*c*33 = 7.0819804e-4 s                (Eq. 16, k > 1)
+      rounds = ceil(ceil(342/2)/16) = 11
+      Talg = 2049*9.24e-7 + 2049*7.0819804e-4*11 = 15.96397 s   (Eq. 17)"""
+    hw = mo.gtx980(3)
+    assert mo.Nw_eq3(8192, 8) == 2049
+    assert mo.wtile_eq4(8, 8) == 14
+    assert mo.w_eq5(8192, 8, 8) == 342
+    assert abs(mo.c_eq15(8, 8, 256, hw) - 1.0724768e-5) < 1e-15
+    t = mo.talg(2, (8192, 8192), 8192, (8, 8, 256, 0), hw)
+    assert abs(t - 15.96397) < 2e-5, t
+
+
+def test_Nw_eq3_equals_exact_row_count():
+    """Eq. 3 with its eps rule is exactly ceil(2T/tT)+1 (reading G2), and both
+    equal the number of non-empty hexagon rows of a brute-force tiling."""
+    for tT in range(2, 34, 2):
+        for T in range(1, 200):
+            assert mo.Nw_eq3(T, tT) == math.ceil(2 * T / tT) + 1
+    for tT in (2, 4, 6, 8):
+        for tS in (1, 2, 3, 5):
+            for T in (1, 2, 5, 8, 13):
+                rows, *_ = hg.analyse(25, T, tS, tT)
+                assert len(rows) == mo.Nw_eq3(T, tT), (tT, tS, T)
+                assert rows == list(range(-1, len(rows) - 1))
+                assert len(list(mo.rows_exact(T, tT))) == len(rows)
+
+
+def test_tiling_is_a_legal_schedule_and_w_counts():
+    """Exact cover (tile_of raises otherwise), dependences only on earlier rows,
+    and the per-row hexagon counts of reading G2."""
+    for tT in (2, 4, 6, 8):
+        for tS in (1, 2, 4, 7):
+            S1, T = 37, 3 * tT + 1
+            rows, w, _, _, _ = hg.analyse(S1, T, tS, tT)
+            wA, wB = mo.w_rows_exact(S1, tS, tT)
+            for m in rows[1:-1]:               # full-height rows
+                assert w[m] == (wA if m % 2 == 0 else wB), (tT, tS, m)
+
+
+def test_exact_footprints_match_enumeration():
+    """Reading G3: an interior hexagon reads tS1+2tT+2 values it did not
+    compute and writes tS1+2tT-2 facets (per unit inner extent)."""
+    for tT in (2, 4, 6, 8, 10):
+        for tS in (1, 2, 3, 6):
+            S1, T = 80, 4 * tT + 3
+            rows, w, reads, writes, tiles = hg.analyse(S1, T, tS, tT)
+            P = 2 * tS + tT
+            for (m, j), pts in tiles.items():
+                ts = {t for t, _ in pts}
+                xs = {x for _, x in pts}
+                if len(pts) != tT * (tS + tT // 2):
+                    continue                    # clipped by time or by the ring
+                if min(xs) < 3 or max(xs) > S1 - 2 or min(ts) < 2 or max(ts) >= T:
+                    continue
+                t0 = min(ts)
+                r, wr = mo.row_io_exact(tS, tT, 0, tT, t0, T)
+                assert reads[(m, j)] == r == tS + 2 * tT + 2, (tT, tS, m, j)
+                assert writes[(m, j)] == wr == tS + 2 * tT - 2, (tT, tS, m, j)
+            assert P == 2 * tS + tT
+
+
+def test_hexagon_area():
+    """Area of the implemented hexagon = tT*(tS1 + tT/2) (reading G1); the
+    paper's wtile = tS+tT-2 row sum (Eq. 9) is tT*(tS1 + tT/2 - 1)."""
+    for tT in range(2, 40, 2):
+        for tS in range(1, 30):
+            assert sum(mo.row_width(t, tS, tT) for t in range(tT)) == tT * (tS + tT // 2)
+            paper = 2 * sum(range(tS, mo.wtile_eq4(tS, tT) + 1, 2))
+            assert paper == tT * (tS + tT // 2 - 1)
+
+
+def test_special_case_wide_vector_units():
+    """if nV >= wtile*tS2 every row takes one Citer, so
+    c = tT*(Citer + tau_sync)."""
+    hw = mo.gtx980(1)
+    hw.nV = 10 ** 9
+    for tT, tS1, tS2 in [(2, 1, 32), (8, 8, 64), (16, 5, 128)]:
+        assert math.isclose(mo.c_eq15(tS1, tT, tS2, hw), tT * (hw.C_iter + hw.tau_sync), rel_tol=1e-12)
+
+
+def test_k_branches():
+    """Eq. 16: k = 1 gives (m'+c)*N2, k > 1 gives m' + k*max(m',c)*N2."""
+    hw = mo.gtx980(2)
+    S, T = (4096, 4096), 1024
+    # a tile with Mtile just under 48 KB -> k = 2; shrink MSM to force k = 1
+    tile = (8, 8, 256, 0)
+    t2 = mo.talg(2, S, T, tile, hw)
+    hw1 = mo.gtx980(2)
+    hw1.MSM = 48 * 1024
+    t1 = mo.talg(2, S, T, tile, hw1)
+    Nw, w = mo.Nw_eq3(T, 8), mo.w_eq5(4096, 8, 8)
+    mi = 256 * (8 + 16)
+    mp = 2 * mi * hw.L + 2 * hw.tau_sync
+    c = mo.c_eq15(8, 8, 256, hw)
+    N2 = math.ceil((4096 + 8) / 256)
+    assert math.isclose(t1, Nw * hw.T_sync + Nw * (mp + c) * N2 * math.ceil(w / 16), rel_tol=1e-12)
+    assert math.isclose(t2, Nw * hw.T_sync + Nw * (mp + 2 * max(mp, c) * N2) * math.ceil(math.ceil(w / 2) / 16),
+                        rel_tol=1e-12)
+
+
+def test_infeasible_and_invalid_tiles():
+    hw = mo.gtx980(2)
+    assert math.isinf(mo.talg(2, (4096, 4096), 64, (16, 64, 1024, 0), hw))   # Mtile > 48 KB
+    assert math.isnan(mo.talg(2, (4096, 4096), 64, (7, 4, 64, 0), hw))       # tT odd
+    assert math.isnan(mo.talg(2, (4096, 4096), 64, (8, 4, 48, 0), hw))       # tS2 not x32
+    assert math.isnan(mo.talg(3, (64, 64, 64), 64, (8, 4, 4, 48), hw))       # tS3 not x32
+
+
+def ideal_compute_bound(S, T, hw):
+    return math.prod(S) * T * hw.C_iter / (hw.nSM * hw.nV)
+
+
+def test_exact_never_beats_ideal_compute_bound():
+    """Every update costs Citer per vector unit: EXACT Talg >= prod(S)*T*Citer/(nSM*nV)."""
+    rnd = random.Random(1)
+    for _ in range(300):
+        kind = rnd.choice([1, 2, 3])
+        hw = mo.gtx980(kind, mo.EXACT)
+        hw.Mblock = 227 * 1024
+        hw.MSM = 228 * 1024
+        S = (rnd.randint(40, 3000), rnd.randint(40, 3000))
+        T = rnd.randint(1, 300)
+        tile = (2 * rnd.randint(1, 16), rnd.randint(1, 30), 32 * rnd.randint(1, 8), 0)
+        t = mo.talg(2, S, T, tile, hw)
+        if math.isfinite(t):
+            assert t >= ideal_compute_bound(S, T, hw) * (1 - 1e-12), (S, T, tile)
+
+
+def test_paper_literal_minimum_is_degenerate():
+    """SURVEY/DESIGN reading M1: at the degenerate tile (2, 1, 640) the literal
+    equations predict less than the ideal compute bound for the Fig. 5 problem,
+    the EXACT geometry does not -- the reason both modes exist."""
+    hw = mo.gtx980(3)
+    S, T = (8192, 8192), 8192
+    ideal = ideal_compute_bound(S, T, hw)
+    assert mo.talg(2, S, T, (2, 1, 640, 0), hw) < ideal
+    hwx = mo.gtx980(3, mo.EXACT)
+    hwx.Mblock, hwx.MSM = 48 * 1024, 96 * 1024
+    assert mo.talg(2, S, T, (2, 1, 640, 0), hwx) >= ideal
+
+
+def test_talg_monotone_in_T():
+    for geom in (mo.PAPER, mo.EXACT):
+        hw = mo.gtx980(2, geom)
+        prev = 0.0
+        for T in range(1, 200, 3):
+            t = mo.talg(2, (1000, 900), T, (8, 6, 64, 0), hw)
+            assert t >= prev
+            prev = t
+
+
+def test_select_tile_small_space():
+    """§6.1: the selector is the exhaustive argmin over Eq. 31's space."""
+    hw = mo.gtx980(2)
+    S, T = (200, 150), 40
+    best, tmin, cands = mo.select_tile(2, S, T, hw, tT_max=16, tS1_max=12, inner_max=256)
+    allv = [(mo.talg(2, S, T, tl, hw), tl) for tl in mo.enumerate_space(2, S, T, hw, tT_max=16,
+                                                                          tS1_max=12, inner_max=256)]
+    allv = [(t, tl) for t, tl in allv if math.isfinite(t)]
+    assert min(allv)[1] == best and min(allv)[0] == tmin
+    assert set(cands) == {tl for t, tl in allv if t <= 1.1 * tmin}
+    assert best in cands
