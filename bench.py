@@ -1,0 +1,296 @@
+#!/usr/bin/env python3
+"""bench.py -- GStencil-updates/s of the HHC stencil path on B200.
+
+A "step" is one pass of the whole hot path (plan, buffer
+setup, every row of hexagons) over one synthetic input: T time steps of the
+config's stencil on its full grid.  N = 1 workload: BASELINE.json configs[1],
+Heat-2D 9-point fp32, 8192^2, T = 1024 (C2).  The tile is the one listed in
+CONFIGS (chosen with model_select_tile + the measured sweep).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config C2] [--impl reference]
+
+Under torchrun (N > 1) the same grid is slab-decomposed along S1 across the
+ranks (strong scaling, ghost exchange over NCCL every time tile) and rank 0
+prints the line; times are the max over ranks of device (CUDA-event) time.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import subprocess
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+CONFIGS = {
+    "C1": dict(kind=1, dims=(256, 256), T=64, tile=(8, 8, 64, 0), threads=0,
+               desc="Jacobi-2D 5-point fp32, 256x256, T=64"),
+    "C2": dict(kind=2, dims=(8192, 8192), T=1024, tile=(16, 20, 512, 0), threads=512,
+               desc="Heat-2D 9-point fp32, 8192x8192, T=1024"),
+    "C3": dict(kind=3, dims=(16384, 16384), T=512, tile=(16, 20, 512, 0), threads=512,
+               desc="Gradient-2D fp32, 16384x16384, T=512"),
+    "C4": dict(kind=4, dims=(512, 512, 512), T=256, tile=(8, 4, 4, 32), threads=0,
+               desc="Heat-3D 7-point fp32, 512^3, T=256"),
+    "C5": dict(kind=5, dims=(768, 768, 768), T=128, tile=(8, 4, 4, 32), threads=0,
+               desc="Laplacian-3D 27-point fp32, 768^3, T=128"),
+}
+DEFAULT_CONFIG = "C2"
+
+# Algorithmic FP32 flops per update of the canonical fused expression
+# (DESIGN.md §Roofline): linear kinds 1 mul + (|N|-1) fma = 2|N|-1; Gradient
+# 19 (sqrt and div counted as one flop each, their SASS sequences are longer).
+FLOPS_PER_UPDATE = {1: 9, 2: 17, 3: 19, 4: 13, 5: 53, 6: 9}
+
+METRIC = "GStencil-updates/s"
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        with open(p) as f:
+            return json.load(f)
+    except OSError:
+        return {}
+
+
+def fp32_peak_tflops(peaks) -> float:
+    """FP32 FMA peak: 148 SMs x 128 lanes x 2 flops x max SM clock."""
+    mhz = float(peaks.get("sm_max_mhz", 1965.0))
+    return 148 * 128 * 2 * mhz * 1e6 / 1e12
+
+
+class ClockSampler:
+    """nvidia-smi clocks/throttle reasons DURING the timed region (B200_PROFILING.md)."""
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int = 0):
+        self.index = index
+        self.proc = None
+        self.path = os.path.join("/tmp", f"hhc_clocks_{os.getpid()}.csv")
+
+    def start(self):
+        try:
+            self.f = open(self.path, "w")
+            self.proc = subprocess.Popen(["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=self.f, stderr=subprocess.DEVNULL)
+        except OSError:
+            self.proc = None
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.25)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except subprocess.TimeoutExpired:
+            self.proc.kill()
+        self.f.close()
+        rows = []
+        for line in open(self.path):
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) >= 9:
+                rows.append(parts)
+        os.unlink(self.path)
+        if not rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["no samples"]}
+        sm = sorted(float(r[1]) for r in rows if r[1].replace(".", "").isdigit())
+        mx = max(float(r[2]) for r in rows if r[2].replace(".", "").isdigit())
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in rows for i in range(4) if r[5 + i].lower() == "active"})
+        load = [s for s in sm if s > 0.5 * mx] or sm
+        return {"sm_mhz": load[len(load) // 2], "sm_max_mhz": mx, "reasons": reasons,
+                "samples": len(rows)}
+
+
+def ncu_traffic(cfg: str):
+    """dram bytes per launch of the dominant kernel from the committed ncu summary."""
+    for name in sorted(os.listdir(os.path.join(ROOT, "profiles")), reverse=True) if os.path.isdir(
+            os.path.join(ROOT, "profiles")) else []:
+        if name.startswith("ncu_summary") and name.endswith(".json"):
+            try:
+                d = json.load(open(os.path.join(ROOT, "profiles", name)))
+            except (OSError, ValueError):
+                continue
+            if cfg in d and d[cfg].get("dram_bytes_per_launch"):
+                return d[cfg]["dram_bytes_per_launch"]
+    return None
+
+
+def cpu_oracle_sample(cfg: dict, seconds: float = 10.0, nthreads: int = 0):
+    """The oracle as it stands (plain mode, all host cores) on a bounded sample
+    of the workload: the full grid for T_s < T steps, T_s sized to ~`seconds`."""
+    import oracle
+    from synth import CONFIG_SEEDS, field
+    name = [k for k, v in CONFIGS.items() if v is cfg][0]
+    a = field(CONFIG_SEEDS[name], cfg["dims"])
+    n_int = math.prod(d - 2 for d in cfg["dims"])
+    t0 = time.perf_counter()
+    oracle.run(cfg["kind"], a, 1, oracle.PLAIN, nthreads=nthreads)
+    one = max(time.perf_counter() - t0, 1e-4)
+    Ts = int(max(1, min(cfg["T"], seconds / one)))
+    t0 = time.perf_counter()
+    oracle.run(cfg["kind"], a, Ts, oracle.PLAIN, nthreads=nthreads)
+    dt = time.perf_counter() - t0
+    cores = nthreads or oracle.max_threads()
+    return {"value": n_int * Ts / dt / 1e9, "unit": METRIC, "cores": cores, "kind": "oracle",
+            "sample": f"full {'x'.join(map(str, cfg['dims']))} grid, {Ts} of {cfg['T']} steps, plain mode, "
+                      f"{dt:.1f} s"}
+
+
+def run_reference(args, cfg, cfgname):
+    """--impl reference: the CPU oracle (the tier's reference arm) on host cores."""
+    import oracle
+    from synth import CONFIG_SEEDS, field
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    a = field(CONFIG_SEEDS[cfgname], cfg["dims"])
+    n_int = math.prod(d - 2 for d in cfg["dims"])
+    t0 = time.perf_counter()
+    oracle.run(cfg["kind"], a, 1, oracle.PLAIN)
+    one = max(time.perf_counter() - t0, 1e-4)
+    budget = 150.0 / max(1, args.steps + args.warmup)      # whole run within a few minutes
+    Ts = int(max(1, min(cfg["T"], budget / one)))
+    for _ in range(args.warmup):
+        oracle.run(cfg["kind"], a, Ts, oracle.PLAIN)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        oracle.run(cfg["kind"], a, Ts, oracle.PLAIN)
+    dt = time.perf_counter() - t0
+    v = n_int * Ts * args.steps / dt / 1e9
+    cores = oracle.max_threads()
+    sample = f"full {'x'.join(map(str, cfg['dims']))} grid, {Ts} of {cfg['T']} steps per step, plain mode"
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": METRIC, "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt / args.steps * 1e3,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f32",
+            "data": "synthetic", "config": {"workload": cfgname + ": " + cfg["desc"]},
+            "cpu_baseline": {"value": v, "unit": METRIC, "cores": cores, "kind": "oracle", "sample": sample},
+            "e2e": {"value": v, "unit": METRIC, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line))
+    return 0
+
+
+def main(argv=None):
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default=DEFAULT_CONFIG, choices=sorted(CONFIGS))
+    ap.add_argument("--impl", default="hhc", choices=["hhc", "reference"])
+    ap.add_argument("--tile", default=None, help="override tile t,s1,s2[,s3]")
+    ap.add_argument("--threads", type=int, default=None)
+    ap.add_argument("--mode", default="fused", choices=["fused", "plain"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    args = ap.parse_args(argv)
+    cfg = CONFIGS[args.config]
+    if args.impl == "reference":
+        return run_reference(args, cfg, args.config)
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    if world > 1 or args.gpus > 1:
+        from paper_conf_ppopp_prajapatirradg17_b200 import dist
+        return dist.bench_main(args, cfg, args.config, CONFIGS)
+    return bench_single(args, cfg, args.config)
+
+
+def bench_single(args, cfg, cfgname):
+    import numpy as np
+    import torch
+
+    import paper_conf_ppopp_prajapatirradg17_b200 as hhc
+    from synth import CONFIG_SEEDS, field
+
+    assert args.warmup >= 3 or os.environ.get("HHC_BENCH_ALLOW_SHORT"), "W >= 3 warm-up steps required"
+    torch.cuda.set_device(0)
+    dev = torch.device("cuda:0")
+    tile = tuple(int(x) for x in args.tile.split(",")) if args.tile else cfg["tile"]
+    tile = tile + (0,) * (4 - len(tile))
+    threads = cfg["threads"] if args.threads is None else args.threads
+    mode = hhc.FUSED if args.mode == "fused" else hhc.PLAIN
+    dims, T, kind = cfg["dims"], cfg["T"], cfg["kind"]
+    n_upd = hhc.updates(dims, T)
+
+    host = field(CONFIG_SEEDS[cfgname], dims)
+    h_in = torch.from_numpy(host).pin_memory()
+    d_in = h_in.to(dev, non_blocking=False)
+    d_out = torch.empty_like(d_in)
+    s = hhc.stencil_create(kind, dims, mode=mode)
+    stream = torch.cuda.current_stream()
+
+    for _ in range(args.warmup):
+        hhc.stencil_run(s, d_in, d_out, T, tile, threads, stream)
+    torch.cuda.synchronize()
+    launches_per_step = hhc.stencil_last_launches(s)
+
+    sampler = ClockSampler(0)
+    sampler.start()
+    time.sleep(0.3)
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    torch.cuda.synchronize()
+    e0.record(stream)
+    for _ in range(args.steps):
+        hhc.stencil_run(s, d_in, d_out, T, tile, threads, stream)
+    e1.record(stream)
+    torch.cuda.synchronize()
+    clocks = sampler.stop()
+    dt = e0.elapsed_time(e1) * 1e-3
+    ms_per_step = dt / args.steps * 1e3
+    value = n_upd * args.steps / dt / 1e9
+
+    # dominant kernel: per-launch device time of the HHC rows (events on the launching stream)
+    ksec, klaunch = hhc.stencil_profile(s, d_in, d_out, T, tile, threads, stream)
+    flops = FLOPS_PER_UPDATE[kind] * n_upd
+    peaks = load_peaks()
+    peak = fp32_peak_tflops(peaks)
+    achieved = flops / ksec / 1e12
+    traffic = ncu_traffic(cfgname)
+    roofline = {"bound": "alu", "achieved": round(achieved, 3), "peak": round(peak, 2), "unit": "TFLOP/s",
+                "frac": round(achieved / peak, 4), "traffic": traffic,
+                "kernel": "hex2d_kernel" if len(dims) == 2 else "hex3d_kernel",
+                "kernel_share_of_step": round(ksec / (dt / args.steps), 4),
+                "kernel_launches_per_step": klaunch,
+                "peak_basis": "148 SM x 128 FP32 lanes x 2 x sm_max_mhz (MEASURED_PEAKS.json)"}
+
+    e2e = None
+    if not args.no_e2e:
+        h_out = torch.empty_like(h_in).pin_memory()
+        hhc.stencil_run_host(s, h_in, h_out, T, tile, threads, stream)
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        for _ in range(args.steps):
+            hhc.stencil_run_host(s, h_in, h_out, T, tile, threads, stream)
+        et = time.perf_counter() - t0
+        nbytes = host.nbytes
+        e2e = {"value": n_upd * args.steps / et / 1e9, "unit": METRIC, "h2d_bytes_per_step": nbytes,
+               "d2h_bytes_per_step": nbytes}
+        # the e2e result must be the same numbers
+        assert torch.equal(h_out, d_out.cpu()), "e2e result differs from device result"
+
+    cpu = None if args.no_cpu_baseline else cpu_oracle_sample(cfg)
+    line = {
+        "metric": METRIC, "value": round(value, 3), "unit": METRIC, "n_gpus": 1, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": round(ms_per_step, 3), "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+        "config": {"workload": cfgname + ": " + cfg["desc"], "tile": list(tile), "threads": threads,
+                   "mode": args.mode, "updates_per_step": n_upd,
+                   "l2": "inputs larger than L2 (plane %d MB > 126 MB)" % (host.nbytes >> 20)
+                   if host.nbytes > 126e6 else "inputs smaller than L2 (launch-bound config)",
+                   "parallelism": "1 GPU, one CTA per hexagonal prism"},
+        "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
+        "gpu_launches": launches_per_step * args.steps,
+    }
+    print(json.dumps(line))
+    hhc.stencil_destroy(s)
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

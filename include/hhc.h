@@ -1,0 +1,185 @@
+/*
+ * hhc.h -- C ABI of the B200 HHC stencil library (libhhc.so).
+ *
+ * Implements the data-parallel hot path of Prajapati et al., "Simple,
+ * Accurate, Analytical Time Modeling and Optimal Tile Size Selection for GPGPU
+ * Stencils" (PPoPP'17).  Citations "P:Lnnn" are PAPER.md lines.
+ *
+ *   stencil_create / stencil_run  -- iterative stencil of Eq. 1
+ *       time-stepped T times under hybrid hexagonal/classic (HHC) tiling
+ *       (§3.1; Fig. 1-2): hexagons of base tS1 and height tT over
+ *       (t, S1), classic time skewing over S2 (and S3), one kernel launch per
+ *       row of hexagons, one thread block per hexagonal prism/slab
+ *       sweeping its sub-tiles sequentially.
+ *   model_predict      -- the analytical execution time Talg, Eqs. 2-30
+ *                         (P:L556-1158).
+ *   model_select_tile  -- Eq. 31 solved by exhaustive enumeration, plus the
+ *                         "within 10% of Talg_min" candidates.
+ *   stencil_run_planes -- one time tile of the slab-decomposed multi-GPU run
+ *                         (BASELINE.json north_star; not in the paper): the
+ *                         ghost exchange is torch.distributed P2P over NCCL in
+ *                         the Python binding, see DESIGN.md §Multi-GPU.
+ *
+ * Conventions (all functions):
+ *   - Sizes are int64.  Arrays are fp32, contiguous, row-major, S1 OUTERMOST,
+ *     the innermost dimension contiguous.
+ *   - dims are the FULL extents including a one-cell fixed (Dirichlet) ring
+ *     (reading R2, "boundary values are given"); the
+ *     interior is [1, S_d-2] and only interior points are updated.
+ *   - Functions return STENCIL_OK (0) or a negative stencil_status.
+ *   - A handle is not thread-safe.  Asynchronous CUDA errors surface as
+ *     STENCIL_ECUDA on the next call on that handle.
+ */
+#ifndef HHC_H
+#define HHC_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    STENCIL_JACOBI2D_5PT = 1,      /* centre + 4 faces, weights 0.2 (reading R1)          */
+    STENCIL_HEAT2D_9PT = 2,        /* 3x3 box, 1/4, 1/8, 1/16                               */
+    STENCIL_GRADIENT2D = 3,        /* non-linear 5-point, kappa = 1/8                       */
+    STENCIL_HEAT3D_7PT = 4,        /* centre + 6 faces, 1/4, 1/8                            */
+    STENCIL_LAPLACIAN3D_27PT = 5,  /* 3x3x3 box, 1/2, 7/128, 3/256, 1/256                   */
+    STENCIL_LAPLACIAN2D_5PT = 6    /* centre + 4 faces, 1/2, 1/8                            */
+} stencil_kind;
+
+typedef enum {
+    STENCIL_OK = 0,
+    STENCIL_EINVAL = -1,   /* bad kind/ndims/dims/pointer/coeffs/T/threads            */
+    STENCIL_ETILE = -2,    /* tile violates Eq. 31's integrality or the smem limit   */
+    STENCIL_ENOMEM = -3,   /* device or host allocation failed                        */
+    STENCIL_ECUDA = -4,    /* a CUDA runtime error (sticky until stencil_destroy)     */
+    STENCIL_ENCCL = -5,    /* reserved: NCCL error (multi-GPU exchange is in Python)  */
+    STENCIL_ENODEV = -6    /* no usable sm_100 device                                 */
+} stencil_status;
+
+typedef enum { STENCIL_MODE_PLAIN = 0, STENCIL_MODE_FUSED = 1 } stencil_mode;
+
+/* Tile sizes: the decision variables of Eq. 31.
+ *   t  = tT  (even, >= 2), s1 = tS1 (>= 1), hexagon base along S1;
+ *   2D: s2 = tS2, a multiple of 32 (inner, contiguous); s3 = 0.
+ *   3D: s2 = tS2 >= 1 (middle), s3 = tS3, a multiple of 32 (inner). */
+typedef struct { int32_t t, s1, s2, s3; } stencil_tile;
+
+/* Table 1 hardware parameters (EH) + C_iter (CSH); Table 2-4. */
+typedef struct {
+    int32_t n_sm;              /* nSM                                                   */
+    int32_t n_v;               /* nV, vector units (FP32 lanes) per SM                  */
+    int32_t mtb_sm;            /* MTBSM, max thread blocks per SM                       */
+    int32_t r_sm;              /* RSM, registers per SM                                 */
+    int64_t m_sm_bytes;        /* MSM, shared memory per SM (bytes)                     */
+    int64_t m_block_bytes;     /* shared memory per thread block (bytes)                */
+    double  L_s_per_word;      /* L, time per 4-byte word of global memory access (s)   */
+    double  tau_sync_s;        /* tau_sync, one block barrier (s)                       */
+    double  T_sync_s;          /* T_sync, one host-GPU synchronisation / launch (s)     */
+    double  C_iter_s;          /* C_iter, one loop-body iteration per vector unit (s)   */
+    int32_t regs_per_thread;   /* 0 = unknown (paper); >0 bounds k in EXACT (Eq. 11)    */
+    int32_t geometry;          /* 0 = PAPER-literal equations, 1 = EXACT (M1) */
+    int32_t threads;           /* threads per block for EXACT k; 0 = library rule      */
+    int32_t max_threads_sm;    /* resident threads per SM (EXACT k); 0 = 2048           */
+    int32_t n_gpus;            /* >1: slab decomposition model (M7)           */
+    double  link_bytes_per_s;  /* per-direction GPU-GPU bandwidth                       */
+    double  link_latency_s;    /* per-message latency                                   */
+} model_hw_params;
+
+typedef struct stencil_s* stencil_t;     /* opaque; owned by the library */
+
+/* Create a handle for one stencil problem on the CURRENT CUDA device.
+ *   kind/ndims must agree (2D kinds: ndims = 2; 3D kinds: ndims = 3);
+ *   dims[ndims] are full extents, each >= 3;
+ *   coeffs == NULL -> the default weights of DESIGN.md R1.  Linear kinds take
+ *   |N| weights in canonical (lexicographic offset) order, optionally followed
+ *   by the constant c of Eq. 1 (ncoeffs = |N| or |N|+1).  Gradient takes {kappa}.
+ *   mode: STENCIL_MODE_PLAIN (separately rounded mul/add) or FUSED (fma),
+ *   see DESIGN.md R4.  The values are copied.  *out receives the handle. */
+int stencil_create(stencil_kind kind, int ndims, const int64_t* dims,
+                   const float* coeffs, int ncoeffs, int mode, stencil_t* out);
+
+/* Release the handle, its scratch plane and its CUDA-graph cache.  NULL is a no-op. */
+void stencil_destroy(stencil_t h);
+
+/* A_T from A_0 = d_in (device pointers, Eq. 1 iterated T times).
+ *   d_in is never written; d_out must not overlap d_in; both hold prod(dims)
+ *   floats.  T >= 0 (T = 0 copies).  threads = 0 -> library rule, else a
+ *   multiple of the tile's column threads (K1) and <= 1024.
+ *   Stream-ordered and asynchronous on cuda_stream (a cudaStream_t, NULL =
+ *   legacy default stream).  The handle owns one scratch plane (allocated on
+ *   first use).  Rows of hexagons are captured once into a CUDA graph per
+ *   (pointers, T, tile, threads, stream) and replayed. */
+int stencil_run(stencil_t h, const float* d_in, float* d_out, int64_t T,
+                stencil_tile tile, int threads, void* cuda_stream);
+
+/* Like stencil_run but with HOST in/out buffers: copies in, runs, copies out,
+ * synchronises (the end-to-end path bench.py's "e2e" measures). */
+int stencil_run_host(stencil_t h, const float* h_in, float* h_out, int64_t T,
+                     stencil_tile tile, int threads, void* cuda_stream);
+
+/* Predicted execution time Talg in seconds (Eqs. 2-30).
+ * dims are full ABI extents (the model uses S = dims-2).  Returns NaN for
+ * invalid arguments and +INFINITY for an infeasible tile (Eq. 31 constraints),
+ * so min-searches skip it. */
+double model_predict(stencil_kind kind, int ndims, const int64_t* dims, int64_t T,
+                     stencil_tile tile, const model_hw_params* hw);
+
+/* Eq. 31 by exhaustive enumeration: *best = argmin Talg (ties:
+ * lexicographically smallest (t, s1, s2, s3)), *best_threads = the library's
+ * threads rule, and the tiles with Talg <= (1+within)*Talg_min written to
+ * cands[0..min(n, cap)) in enumeration order, *n_cands = n (may exceed cap).
+ * Search space: DESIGN.md reading M6.  Returns STENCIL_ETILE if no tile is
+ * feasible. */
+int model_select_tile(stencil_kind kind, int ndims, const int64_t* dims, int64_t T,
+                      const model_hw_params* hw, double within,
+                      stencil_tile* best, int* best_threads,
+                      stencil_tile* cands, int cap, int* n_cands);
+
+/* Shared-memory bytes and threads the kernel uses for (ndims, tile, threads);
+ * 0 / error if the tile is invalid.  Lets callers and the model agree on Mtile. */
+int stencil_tile_resources(int ndims, stencil_tile tile, int threads,
+                           int64_t* smem_bytes, int* block_threads, int* regs_per_thread);
+
+/* Launch geometry of a run: number of hexagon rows (kernel launches, Nw) and
+ * the number of thread blocks of phase-A and phase-B rows (w(i), Eq. 5). */
+int stencil_plan_info(int ndims, const int64_t* dims, int64_t T, stencil_tile tile,
+                      int64_t* n_rows, int64_t* w_a, int64_t* w_b, int64_t* n_sub);
+
+/* Calibration micro-benchmarks (§5.2) on the current device.
+ *   which: 0 = L (s per word, all SMs streaming), 1 = tau_sync (s per block
+ *   barrier), 2 = T_sync (s per back-to-back launch), 3 = C_iter of `kind`
+ *   at `tile` (compute-only kernel with global<->shared transfers removed).
+ *   *value receives the measurement. */
+int stencil_microbench(int which, stencil_kind kind, int ndims, const int64_t* dims,
+                       int64_t T, stencil_tile tile, int threads, double* value);
+
+/* One time tile of the multi-GPU slab path, also usable
+ * alone: run T steps on a domain of `rows` x dims[1] (x dims[2]) whose level 0
+ * (ring included) is in plane0 (device, read AND overwritten as scratch);
+ * plane1 (device, same size, no overlap) receives the ring, then serves as the
+ * second parity plane.  The result A_T is left in plane0 if T is even, plane1
+ * if T is odd.  Inner extents come from the handle; rows may differ from
+ * dims[0] (ghost-extended slabs).  Stream-ordered like stencil_run. */
+int stencil_run_planes(stencil_t h, int64_t rows, float* plane0, float* plane1, int64_t T,
+                       stencil_tile tile, int threads, void* cuda_stream);
+
+/* Measurement helper (bench.py roofline): run like stencil_run but without the
+ * CUDA graph, with a CUDA event pair around every hexagon-row launch on
+ * cuda_stream; synchronises and returns the summed device time of the HHC
+ * kernel launches (*kernel_seconds) and their number (*kernel_launches). */
+int stencil_profile(stencil_t h, const float* d_in, float* d_out, int64_t T, stencil_tile tile,
+                    int threads, void* cuda_stream, double* kernel_seconds, int64_t* kernel_launches);
+
+/* Human-readable status. */
+const char* stencil_strerror(int status);
+
+/* Number of kernel launches the last stencil_run / stencil_run_planes on h
+ * issued (for the bench's gpu_launches claim). */
+int64_t stencil_last_launches(stencil_t h);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* HHC_H */

@@ -1,0 +1,525 @@
+// hhc_api.cu -- the C ABI of include/hhc.h: handles, planning (§8(a) a1-a3),
+// buffer roles (a2), the row-of-hexagons launch sequence captured as a CUDA
+// graph (a3), and host-buffer runs for the end-to-end measurement.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdlib>
+#include <cstring>
+#include <vector>
+
+#include "hhc_internal.h"
+
+using namespace hhc;
+
+namespace {
+
+int kind_ndims_host(int kind) {
+    switch (kind) {
+    case STENCIL_JACOBI2D_5PT: case STENCIL_HEAT2D_9PT: case STENCIL_GRADIENT2D:
+    case STENCIL_LAPLACIAN2D_5PT: return 2;
+    case STENCIL_HEAT3D_7PT: case STENCIL_LAPLACIAN3D_27PT: return 3;
+    default: return 0;
+    }
+}
+
+// Default weights (reading R1) by number of non-zero offset components.
+float default_weight(int kind, int nz) {
+    switch (kind) {
+    case STENCIL_JACOBI2D_5PT: return 0.2f;
+    case STENCIL_LAPLACIAN2D_5PT: return nz == 0 ? 0.5f : 0.125f;
+    case STENCIL_HEAT2D_9PT: return nz == 0 ? 0.25f : (nz == 1 ? 0.125f : 0.0625f);
+    case STENCIL_HEAT3D_7PT: return nz == 0 ? 0.25f : 0.125f;
+    case STENCIL_LAPLACIAN3D_27PT:
+        return nz == 0 ? 0.5f : nz == 1 ? 7.0f / 128.0f : nz == 2 ? 3.0f / 256.0f : 1.0f / 256.0f;
+    default: return 0.0f;
+    }
+}
+
+bool in_nb(int kind, int nz) {
+    return (kind == STENCIL_HEAT2D_9PT || kind == STENCIL_LAPLACIAN3D_27PT) ? true : nz <= 1;
+}
+
+
+struct RowPlan {
+    int m;
+    int64_t t0, xbase;
+    int tau_lo, tau_hi;
+    int w, n2, n3, J;
+};
+
+int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
+
+}  // namespace
+
+struct RunSpec {
+    int planes_mode;          // 0: stencil_run (in -> out); 1: stencil_run_planes
+    const float* a;           // in  | plane0
+    float* b;                 // out | plane1
+    int64_t dims[3];
+    int64_t T;
+    stencil_tile tile;
+    int G, thr;
+};
+
+struct GraphEntry {
+    RunSpec spec;
+    cudaGraphExec_t exec;
+    int64_t launches;
+    uint64_t last_use;
+};
+
+struct stencil_s {
+    int kind = 0, ndims = 0, mode = 0;
+    int64_t dims[3] = {1, 1, 1};
+    int npts = 0;
+    float w[kMaxPts] = {};
+    float c = 0.0f, kappa = 0.125f;
+    bool has_c = false;
+    int device = 0, nsm = 148, smem_optin = 227 * 1024;
+    float* scratch = nullptr;
+    unsigned* flags = nullptr;
+    int64_t flags_n = 0;
+    float* h_in_dev = nullptr;   // stencil_run_host device buffers
+    float* h_out_dev = nullptr;
+    int sticky = 0;
+    int64_t last_launches = 0;
+    cudaStream_t cap_stream = nullptr;
+    std::vector<GraphEntry> graphs;
+    uint64_t use_clock = 0;
+    int compute_only = 0;
+
+    int64_t nelem() const { return dims[0] * dims[1] * dims[2]; }
+};
+
+extern "C" const char* stencil_strerror(int status) {
+    switch (status) {
+    case STENCIL_OK: return "ok";
+    case STENCIL_EINVAL: return "invalid argument";
+    case STENCIL_ETILE: return "invalid or infeasible tile";
+    case STENCIL_ENOMEM: return "out of memory";
+    case STENCIL_ECUDA: return "CUDA error";
+    case STENCIL_ENCCL: return "NCCL error";
+    case STENCIL_ENODEV: return "no usable sm_100 device";
+    default: return "unknown status";
+    }
+}
+
+static int cuda_fail(stencil_t h, cudaError_t e) {
+    if (e == cudaSuccess) return STENCIL_OK;
+    if (h) h->sticky = STENCIL_ECUDA;
+    return e == cudaErrorMemoryAllocation ? STENCIL_ENOMEM : STENCIL_ECUDA;
+}
+
+extern "C" int stencil_create(stencil_kind kind, int ndims, const int64_t* dims, const float* coeffs,
+                              int ncoeffs, int mode, stencil_t* out) {
+    if (!out || !dims) return STENCIL_EINVAL;
+    *out = nullptr;
+    const int D = kind_ndims_host(kind);
+    if (D == 0 || D != ndims) return STENCIL_EINVAL;
+    if (mode != STENCIL_MODE_PLAIN && mode != STENCIL_MODE_FUSED) return STENCIL_EINVAL;
+    for (int d = 0; d < ndims; ++d)
+        if (dims[d] < 3) return STENCIL_EINVAL;
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess) return STENCIL_ENODEV;
+    cudaDeviceProp prop;
+    if (cudaGetDeviceProperties(&prop, dev) != cudaSuccess) return STENCIL_ENODEV;
+    if (prop.major < 10) return STENCIL_ENODEV;   // sm_100a code only
+    stencil_s* h = new stencil_s();
+    h->kind = kind; h->ndims = ndims; h->mode = mode;
+    for (int d = 0; d < ndims; ++d) h->dims[d] = dims[d];
+    h->device = dev;
+    h->nsm = prop.multiProcessorCount;
+    h->smem_optin = (int)prop.sharedMemPerBlockOptin;
+    if (kind == STENCIL_GRADIENT2D) {
+        h->npts = 5;
+        if (coeffs) {
+            if (ncoeffs != 1) { delete h; return STENCIL_EINVAL; }
+            h->kappa = coeffs[0];
+        }
+    } else {
+        int n = 0;
+        for (int d1 = -1; d1 <= 1; ++d1)
+            for (int d2 = -1; d2 <= 1; ++d2)
+                for (int d3 = (D == 3 ? -1 : 0); d3 <= (D == 3 ? 1 : 0); ++d3) {
+                    const int nz = (d1 != 0) + (d2 != 0) + (d3 != 0);
+                    if (!in_nb(kind, nz)) continue;
+                    h->w[n++] = default_weight(kind, nz);
+                }
+        h->npts = n;
+        if (coeffs) {
+            if (ncoeffs != n && ncoeffs != n + 1) { delete h; return STENCIL_EINVAL; }
+            for (int j = 0; j < n; ++j) h->w[j] = coeffs[j];
+            if (ncoeffs == n + 1 && coeffs[n] != 0.0f) { h->has_c = true; h->c = coeffs[n]; }
+        }
+    }
+    if (cudaStreamCreateWithFlags(&h->cap_stream, cudaStreamNonBlocking) != cudaSuccess) {
+        delete h;
+        return STENCIL_ECUDA;
+    }
+    *out = h;
+    return STENCIL_OK;
+}
+
+extern "C" void stencil_destroy(stencil_t h) {
+    if (!h) return;
+    for (auto& g : h->graphs) cudaGraphExecDestroy(g.exec);
+    if (h->scratch) cudaFree(h->scratch);
+    if (h->flags) cudaFree(h->flags);
+    if (h->h_in_dev) cudaFree(h->h_in_dev);
+    if (h->h_out_dev) cudaFree(h->h_out_dev);
+    if (h->cap_stream) cudaStreamDestroy(h->cap_stream);
+    delete h;
+}
+
+// ---- tile validation (§8(b) validation rules; Eq. 31 integrality)
+static int check_tile(int ndims, stencil_tile t, int threads, int smem_limit, int* G_out, int* thr_out) {
+    if (t.t < 2 || (t.t & 1) || t.s1 < 1) return STENCIL_ETILE;
+    if (ndims == 2) {
+        if (t.s2 < 32 || t.s2 % 32) return STENCIL_ETILE;
+    } else {
+        if (t.s2 < 1 || t.s3 < 32 || t.s3 % 32) return STENCIL_ETILE;
+    }
+    if (t.t > 1024 || t.s1 > 4096 || t.s2 > 8192 || (ndims == 3 && t.s3 > 4096)) return STENCIL_ETILE;
+    const int base = column_threads(ndims, t.s2, t.s3);
+    if (base > 512) return STENCIL_ETILE;
+    int G;
+    if (threads == 0) {
+        G = base <= 256 ? std::max(1, std::min(4, 256 / base)) : 1;
+    } else {
+        if (threads < 0 || threads > 512 || threads % base) return STENCIL_EINVAL;
+        G = threads / base;
+    }
+    const int64_t sm = smem_bytes(ndims, t.t, t.s1, t.s2, t.s3);
+    if (sm > smem_limit) return STENCIL_ETILE;
+    *G_out = G;
+    *thr_out = base * G;
+    return STENCIL_OK;
+}
+
+extern "C" int stencil_tile_resources(int ndims, stencil_tile tile, int threads, int64_t* smem,
+                                      int* block_threads, int* regs) {
+    if (ndims != 2 && ndims != 3) return STENCIL_EINVAL;
+    int G, thr;
+    const int rc = check_tile(ndims, tile, threads, 227 * 1024, &G, &thr);
+    if (rc) return rc;
+    if (smem) *smem = smem_bytes(ndims, tile.t, tile.s1, tile.s2, tile.s3);
+    if (block_threads) *block_threads = thr;
+    if (regs) *regs = 0;
+    return STENCIL_OK;
+}
+
+// ---- planning (a1, a3): rows m = -1 .. Nw-2 (reading G2)
+static void plan_rows(int ndims, const int64_t* dims, int64_t T, stencil_tile t, std::vector<RowPlan>& rows) {
+    rows.clear();
+    const int64_t S1i = dims[0] - 2;
+    const int h = t.t / 2;
+    const int P = 2 * t.s1 + t.t;
+    const int64_t Nw = cdiv(2 * T, t.t) + 1;
+    const int64_t wA = cdiv(S1i + h, P);
+    const int64_t wB = S1i > t.s1 ? cdiv(S1i - t.s1, P) : 0;
+    for (int64_t m = -1; m <= Nw - 2; ++m) {
+        RowPlan r;
+        r.m = (int)m;
+        r.t0 = 1 + m * h;
+        r.tau_lo = (int)std::max<int64_t>(0, 1 - r.t0);
+        r.tau_hi = (int)std::min<int64_t>(t.t, T - r.t0 + 1);
+        const bool A = (m % 2 == 0);
+        r.xbase = A ? 1 : 1 + t.s1 + h;
+        r.w = (int)(A ? wA : wB);
+        const int nlev = r.tau_hi - r.tau_lo;
+        if (ndims == 2) {
+            r.n2 = (int)cdiv(dims[1] - 2 + nlev - 1, t.s2);
+            r.n3 = 1;
+        } else {
+            r.n2 = (int)cdiv(dims[1] - 2 + nlev - 1, t.s2);
+            r.n3 = (int)cdiv(dims[2] - 2 + nlev - 1, t.s3);
+        }
+        r.J = 1;
+        if (nlev > 0 && r.w > 0) rows.push_back(r);
+    }
+}
+
+extern "C" int stencil_plan_info(int ndims, const int64_t* dims, int64_t T, stencil_tile tile,
+                                 int64_t* n_rows, int64_t* w_a, int64_t* w_b, int64_t* n_sub) {
+    if ((ndims != 2 && ndims != 3) || !dims || T < 1) return STENCIL_EINVAL;
+    int G, thr;
+    const int rc = check_tile(ndims, tile, 0, 1 << 30, &G, &thr);
+    if (rc) return rc;
+    std::vector<RowPlan> rows;
+    plan_rows(ndims, dims, T, tile, rows);
+    const int64_t S1i = dims[0] - 2;
+    const int P = 2 * tile.s1 + tile.t;
+    if (n_rows) *n_rows = cdiv(2 * T, tile.t) + 1;
+    if (w_a) *w_a = cdiv(S1i + tile.t / 2, P);
+    if (w_b) *w_b = S1i > tile.s1 ? cdiv(S1i - tile.s1, P) : 0;
+    if (n_sub) {
+        int64_t ns = 0;
+        for (auto& r : rows) ns = std::max<int64_t>(ns, (int64_t)r.n2 * r.n3);
+        *n_sub = ns;
+    }
+    return STENCIL_OK;
+}
+
+// Enqueue the hexagon rows (a3) for a domain of extents dims whose level 0 is
+// in plane0 (ring included) and whose ring is also present in plane1; the
+// result (level T) lands in plane[T & 1].  Ring values are read from `ring`.
+static int enqueue_rows(stencil_t h, const int64_t* dims, const float* ring, float* plane0, float* plane1,
+                        int64_t T, stencil_tile tile, int G, int thr, cudaStream_t s, int64_t* launches,
+                        std::vector<cudaEvent_t>* evs = nullptr) {
+    std::vector<RowPlan> rows;
+    plan_rows(h->ndims, dims, T, tile, rows);
+    hex_kernel_t k = get_hex_kernel(h->ndims, h->kind, h->mode, h->has_c);
+    if (!k) return STENCIL_EINVAL;
+    const int64_t smem = smem_bytes(h->ndims, tile.t, tile.s1, tile.s2, tile.s3);
+    cudaError_t e = cudaFuncSetAttribute((const void*)k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return cuda_fail(h, e);
+    int64_t nl = 0;
+    // 3D: thread blocks per slab J (pipelined along S2, flags in global memory);
+    // all blocks of a launch must be co-resident when J > 1 (no deadlock).
+    if (h->ndims == 3) {
+        int occ = 1;
+        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, (const void*)k, thr, (size_t)smem);
+        if (e != cudaSuccess) return cuda_fail(h, e);
+        occ = std::max(occ, 1);
+        int64_t need = 0;
+        const char* envJ = getenv("HHC_J");
+        for (auto& r : rows) {
+            const int cap = std::max(1, h->nsm * occ / std::max(r.w, 1));
+            int J = std::max(1, std::min(r.n2, cap));
+            if (envJ) J = std::max(1, std::min({atoi(envJ), r.n2, cap}));
+            r.J = J;
+            if (J > 1) need = std::max<int64_t>(need, (int64_t)r.w * r.n2);
+        }
+        if (need > h->flags_n) {
+            if (h->flags) cudaFree(h->flags);
+            h->flags = nullptr;
+            h->flags_n = 0;
+            e = cudaMalloc(&h->flags, need * sizeof(unsigned));
+            if (e != cudaSuccess) return cuda_fail(h, e);
+            h->flags_n = need;
+        }
+        if (need > 0) {
+            e = cudaMemsetAsync(h->flags, 0, need * sizeof(unsigned), s);
+            if (e != cudaSuccess) return cuda_fail(h, e);
+        }
+    }
+    HexParams p;
+    memset(&p, 0, sizeof(p));
+    p.in = ring;
+    p.plane[0] = plane0;
+    p.plane[1] = plane1;
+    p.S1 = dims[0]; p.S2 = dims[1]; p.S3 = h->ndims == 3 ? dims[2] : 1;
+    p.T = T;
+    p.tT = tile.t; p.tS1 = tile.s1; p.tS2 = tile.s2; p.tS3 = h->ndims == 3 ? tile.s3 : 0;
+    p.G = G;
+    p.P = 2 * tile.s1 + tile.t;
+    for (int j = 0; j < kMaxPts; ++j) p.w[j] = h->w[j];
+    p.c = h->c;
+    p.kappa = h->kappa;
+    p.flags = h->flags;
+    p.compute_only = h->compute_only;
+    for (auto& r : rows) {
+        p.t0 = r.t0; p.xbase = r.xbase; p.tau_lo = r.tau_lo; p.tau_hi = r.tau_hi;
+        p.n2 = r.n2; p.n3 = r.n3; p.J = r.J;
+        p.epoch = (unsigned)(r.m + 2) << 16;
+        void* args[] = {&p};
+        if (evs) {
+            cudaEvent_t a, b;
+            cudaEventCreate(&a);
+            cudaEventCreate(&b);
+            evs->push_back(a);
+            evs->push_back(b);
+            cudaEventRecord(a, s);
+        }
+        e = cudaLaunchKernel((const void*)k, dim3((unsigned)(r.w * r.J)), dim3(thr), args, (size_t)smem, s);
+        if (e != cudaSuccess) return cuda_fail(h, e);
+        if (evs) cudaEventRecord(evs->back(), s);
+        ++nl;
+    }
+    *launches = nl;
+    return STENCIL_OK;
+}
+
+static int enqueue_spec(stencil_t h, const RunSpec& r, cudaStream_t s, int64_t* launches) {
+    const int64_t n = r.dims[0] * r.dims[1] * r.dims[2];
+    int64_t nl = 0, nrows = 0;
+    int rc;
+    if (r.planes_mode == 0) {
+        float* plane[2];
+        plane[r.T & 1] = r.b;
+        plane[1 - (r.T & 1)] = h->scratch;
+        // a2: level 0 in plane 0, the fixed ring in plane 1 (readings R2/R3)
+        launch_copy_full(r.a, plane[0], n, s); ++nl;
+        launch_copy_ring(r.a, plane[1], r.dims[0], r.dims[1], r.dims[2], s); ++nl;
+        rc = enqueue_rows(h, r.dims, r.a, plane[0], plane[1], r.T, r.tile, r.G, r.thr, s, &nrows);
+    } else {
+        float* p0 = const_cast<float*>(r.a);
+        launch_copy_ring(p0, r.b, r.dims[0], r.dims[1], r.dims[2], s); ++nl;
+        rc = enqueue_rows(h, r.dims, p0, p0, r.b, r.T, r.tile, r.G, r.thr, s, &nrows);
+    }
+    *launches = nl + nrows;
+    return rc;
+}
+
+static bool same_spec(const RunSpec& x, const RunSpec& y) {
+    return x.planes_mode == y.planes_mode && x.a == y.a && x.b == y.b && x.dims[0] == y.dims[0] &&
+           x.dims[1] == y.dims[1] && x.dims[2] == y.dims[2] && x.T == y.T && x.tile.t == y.tile.t &&
+           x.tile.s1 == y.tile.s1 && x.tile.s2 == y.tile.s2 && x.tile.s3 == y.tile.s3 && x.G == y.G &&
+           x.thr == y.thr;
+}
+
+// Run a spec through the CUDA-graph cache (captured once per spec, replayed).
+static int run_spec(stencil_t h, const RunSpec& r, cudaStream_t s) {
+    const bool use_graph = getenv("HHC_NO_GRAPH") == nullptr && !h->compute_only;
+    if (!use_graph) {
+        int64_t nl = 0;
+        int rc = enqueue_spec(h, r, s, &nl);
+        h->last_launches = nl;
+        if (rc) return rc;
+        return cuda_fail(h, cudaGetLastError());
+    }
+    for (auto& g : h->graphs) {
+        if (same_spec(g.spec, r)) {
+            g.last_use = ++h->use_clock;
+            h->last_launches = g.launches;
+            return cuda_fail(h, cudaGraphLaunch(g.exec, s));
+        }
+    }
+    // capture on the private stream, then launch on the caller's stream
+    cudaGraph_t graph = nullptr;
+    cudaError_t e = cudaStreamBeginCapture(h->cap_stream, cudaStreamCaptureModeThreadLocal);
+    if (e != cudaSuccess) return cuda_fail(h, e);
+    int64_t nl = 0;
+    int rc = enqueue_spec(h, r, h->cap_stream, &nl);
+    e = cudaStreamEndCapture(h->cap_stream, &graph);
+    if (rc) { if (graph) cudaGraphDestroy(graph); return rc; }
+    if (e != cudaSuccess) return cuda_fail(h, e);
+    cudaGraphExec_t exec = nullptr;
+    e = cudaGraphInstantiate(&exec, graph, 0);
+    cudaGraphDestroy(graph);
+    if (e != cudaSuccess) return cuda_fail(h, e);
+    if (h->graphs.size() >= 32) {
+        auto it = std::min_element(h->graphs.begin(), h->graphs.end(),
+                                   [](const GraphEntry& a, const GraphEntry& b) { return a.last_use < b.last_use; });
+        cudaGraphExecDestroy(it->exec);
+        h->graphs.erase(it);
+    }
+    h->graphs.push_back(GraphEntry{r, exec, nl, ++h->use_clock});
+    h->last_launches = nl;
+    return cuda_fail(h, cudaGraphLaunch(exec, s));
+}
+
+extern "C" int stencil_run(stencil_t h, const float* d_in, float* d_out, int64_t T, stencil_tile tile,
+                           int threads, void* cuda_stream) {
+    if (!h) return STENCIL_EINVAL;
+    if (h->sticky) return h->sticky;
+    if (!d_in || !d_out || T < 0) return STENCIL_EINVAL;
+    const int64_t n = h->nelem();
+    if (d_out < d_in + n && d_in < d_out + n) return STENCIL_EINVAL;   // overlap
+    cudaStream_t s = (cudaStream_t)cuda_stream;
+    cudaSetDevice(h->device);
+    if (T == 0) {
+        h->last_launches = 1;
+        launch_copy_full(d_in, d_out, n, s);
+        return cuda_fail(h, cudaGetLastError());
+    }
+    RunSpec r;
+    int rc = check_tile(h->ndims, tile, threads, h->smem_optin, &r.G, &r.thr);
+    if (rc) return rc;
+    if (!h->scratch) {
+        cudaError_t e = cudaMalloc(&h->scratch, n * sizeof(float));
+        if (e != cudaSuccess) { h->scratch = nullptr; return STENCIL_ENOMEM; }
+    }
+    r.planes_mode = 0; r.a = d_in; r.b = d_out;
+    for (int d = 0; d < 3; ++d) r.dims[d] = h->dims[d];
+    r.T = T; r.tile = tile;
+    if (h->ndims == 2) r.tile.s3 = 0;
+    return run_spec(h, r, s);
+}
+
+extern "C" int stencil_run_planes(stencil_t h, int64_t rows, float* plane0, float* plane1, int64_t T,
+                                  stencil_tile tile, int threads, void* cuda_stream) {
+    if (!h) return STENCIL_EINVAL;
+    if (h->sticky) return h->sticky;
+    if (!plane0 || !plane1 || T < 1 || rows < 3) return STENCIL_EINVAL;
+    RunSpec r;
+    int rc = check_tile(h->ndims, tile, threads, h->smem_optin, &r.G, &r.thr);
+    if (rc) return rc;
+    cudaSetDevice(h->device);
+    r.planes_mode = 1; r.a = plane0; r.b = plane1;
+    r.dims[0] = rows; r.dims[1] = h->dims[1]; r.dims[2] = h->dims[2];
+    const int64_t n = r.dims[0] * r.dims[1] * r.dims[2];
+    if (plane1 < plane0 + n && plane0 < plane1 + n) return STENCIL_EINVAL;
+    r.T = T; r.tile = tile;
+    if (h->ndims == 2) r.tile.s3 = 0;
+    return run_spec(h, r, (cudaStream_t)cuda_stream);
+}
+
+extern "C" int stencil_run_host(stencil_t h, const float* h_in, float* h_out, int64_t T, stencil_tile tile,
+                                int threads, void* cuda_stream) {
+    if (!h || !h_in || !h_out) return STENCIL_EINVAL;
+    if (h->sticky) return h->sticky;
+    const int64_t n = h->nelem();
+    cudaStream_t s = (cudaStream_t)cuda_stream;
+    cudaSetDevice(h->device);
+    if (!h->h_in_dev) {
+        if (cudaMalloc(&h->h_in_dev, n * sizeof(float)) != cudaSuccess) { h->h_in_dev = nullptr; return STENCIL_ENOMEM; }
+        if (cudaMalloc(&h->h_out_dev, n * sizeof(float)) != cudaSuccess) { h->h_out_dev = nullptr; return STENCIL_ENOMEM; }
+    }
+    cudaError_t e = cudaMemcpyAsync(h->h_in_dev, h_in, n * sizeof(float), cudaMemcpyHostToDevice, s);
+    if (e != cudaSuccess) return cuda_fail(h, e);
+    int rc = stencil_run(h, h->h_in_dev, h->h_out_dev, T, tile, threads, cuda_stream);
+    if (rc) return rc;
+    e = cudaMemcpyAsync(h_out, h->h_out_dev, n * sizeof(float), cudaMemcpyDeviceToHost, s);
+    if (e != cudaSuccess) return cuda_fail(h, e);
+    return cuda_fail(h, cudaStreamSynchronize(s));
+}
+
+extern "C" int64_t stencil_last_launches(stencil_t h) { return h ? h->last_launches : 0; }
+
+extern "C" int stencil_profile(stencil_t h, const float* d_in, float* d_out, int64_t T, stencil_tile tile,
+                               int threads, void* cuda_stream, double* kernel_seconds, int64_t* kernel_launches) {
+    if (!h || !kernel_seconds || !kernel_launches) return STENCIL_EINVAL;
+    if (h->sticky) return h->sticky;
+    if (!d_in || !d_out || T < 1) return STENCIL_EINVAL;
+    int G, thr;
+    int rc = check_tile(h->ndims, tile, threads, h->smem_optin, &G, &thr);
+    if (rc) return rc;
+    const int64_t n = h->nelem();
+    if (!h->scratch) {
+        if (cudaMalloc(&h->scratch, n * sizeof(float)) != cudaSuccess) { h->scratch = nullptr; return STENCIL_ENOMEM; }
+    }
+    cudaStream_t s = (cudaStream_t)cuda_stream;
+    cudaSetDevice(h->device);
+    float* plane[2];
+    plane[T & 1] = d_out;
+    plane[1 - (T & 1)] = h->scratch;
+    launch_copy_full(d_in, plane[0], n, s);
+    launch_copy_ring(d_in, plane[1], h->dims[0], h->dims[1], h->dims[2], s);
+    std::vector<cudaEvent_t> evs;
+    int64_t nl = 0;
+    rc = enqueue_rows(h, h->dims, d_in, plane[0], plane[1], T, tile, G, thr, s, &nl, &evs);
+    if (rc == STENCIL_OK) rc = cuda_fail(h, cudaStreamSynchronize(s));
+    double tot = 0.0;
+    for (size_t i = 0; i + 1 < evs.size(); i += 2) {
+        float ms = 0.0f;
+        if (rc == STENCIL_OK) cudaEventElapsedTime(&ms, evs[i], evs[i + 1]);
+        tot += ms * 1e-3;
+    }
+    for (auto ev : evs) cudaEventDestroy(ev);
+    *kernel_seconds = tot;
+    *kernel_launches = (int64_t)(evs.size() / 2);
+    return rc;
+}
+
+extern "C" int stencil_microbench(int which, stencil_kind kind, int ndims, const int64_t* dims, int64_t T,
+                                  stencil_tile tile, int threads, double* value) {
+    if (!value) return STENCIL_EINVAL;
+    return run_microbench(which, kind, ndims, dims, T, tile, threads, value);
+}
+
+namespace hhc {
+void set_compute_only(stencil_t h, int on) { if (h) h->compute_only = on; }
+}

@@ -1,0 +1,59 @@
+// hhc_internal.h -- host/device structures shared by the library's own .cu/.cpp
+// files (never by the oracle).  See DESIGN.md §Kernels for the layouts.
+#pragma once
+#include <stdint.h>
+
+#include "../../include/hhc.h"
+
+namespace hhc {
+
+constexpr int kColsPerThread = 4;   // B: inner-dimension columns per thread (float4)
+constexpr int kMaxPts = 27;
+
+// Kernel parameters for one launch = one row of hexagons.
+struct HexParams {
+    const float* in;        // A_0 (ring values are read from here)
+    float* plane[2];        // plane[t & 1] holds level t (two-plane storage, reading R3)
+    int64_t S1, S2, S3;     // full extents (S3 = 1 in 2D)
+    int64_t T;
+    int tT, tS1, tS2, tS3;
+    int G;                  // x-groups of threads (threads = column threads * G)
+    int P;                  // pitch 2 tS1 + tT (Eq. 5)
+    int64_t t0;             // level of tau = 0 of this row: 1 + m tT/2
+    int64_t xbase;          // x0 of hexagon 0 of this row (reading G2)
+    int tau_lo, tau_hi;     // levels of the row clipped to [1, T]
+    int n2, n3;             // sub-tiles along S2 (and S3 in 3D)
+    int J;                  // 3D: thread blocks per hexagonal slab (pipelined along S2)
+    unsigned* flags;        // 3D, J > 1: progress flags [w][n2]
+    unsigned epoch;         // flag value base for this row
+    float w[kMaxPts];       // weights in canonical order (reading R4)
+    float c;                // Eq. 1 constant
+    float kappa;            // Gradient-2D
+    int compute_only;       // K4: skip all global<->shared transfers (Citer micro-benchmark)
+};
+
+// Shared-memory bytes of the HHC kernels (DESIGN.md §Kernels K1/K2): two parity
+// planes in skewed coordinates plus a double-buffered skewed face.
+inline int64_t smem_bytes(int ndims, int tT, int tS1, int tS2, int tS3) {
+    const int64_t NX = tS1 + tT + 2;
+    if (ndims == 2) return 4 * (2 * NX * (tS2 + 4) + 2 * (int64_t)tT * NX * 2);
+    return 4 * (2 * NX * (tS2 + 2) * (tS3 + 4) + 2 * (int64_t)tT * NX * (tS2 + 2) * 2);
+}
+
+inline int column_threads(int ndims, int tS2, int tS3) {
+    return ndims == 2 ? tS2 / kColsPerThread : (tS3 / kColsPerThread) * tS2;
+}
+
+typedef void (*hex_kernel_t)(HexParams);
+hex_kernel_t get_hex_kernel(int ndims, int kind, int mode, bool has_c);
+int hex_kernel_regs(int ndims, int kind, int mode, bool has_c);
+void launch_copy_ring(const float* in, float* out, int64_t S1, int64_t S2, int64_t S3, void* stream);
+void launch_copy_full(const float* in, float* out, int64_t n, void* stream);
+
+void set_compute_only(stencil_t h, int on);
+
+// Microbenchmarks (microbench.cu)
+int run_microbench(int which, int kind, int ndims, const int64_t* dims, int64_t T,
+                   stencil_tile tile, int threads, double* value);
+
+}  // namespace hhc

@@ -1,0 +1,151 @@
+// microbench.cu -- calibration micro-benchmarks of PAPER.md §5.2,
+// re-measured on B200 (§8(a) a12):
+//   0: L        -- time per 4-byte word of global memory access, all SMs
+//                  streaming a copy larger than L2 (device-level, Table 3 units
+//                  converted to s/word, reading M5);
+//   1: tau_sync -- one block barrier (__syncthreads) with `threads` threads;
+//   2: T_sync   -- one back-to-back kernel launch inside a CUDA graph (our runs
+//                  replay a graph of row launches);
+//   3: C_iter   -- the HHC kernel of `kind` with all global<->shared transfers
+//                  removed, divided by the EXACT model's
+//                  iteration count (Talg with C_iter = 1, L = tau = T_sync = 0).
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <vector>
+
+#include "hhc_internal.h"
+
+namespace hhc {
+
+__global__ void mb_copy_kernel(const float4* __restrict__ a, float4* __restrict__ b, int64_t n4) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n4; i += (int64_t)gridDim.x * blockDim.x)
+        b[i] = __ldcs(a + i);
+}
+
+__global__ void mb_sync_kernel(int iters, float* sink) {
+    float v = threadIdx.x;
+    for (int i = 0; i < iters; ++i) {
+        __syncthreads();
+        v = v * 1.0000001f + 1.0f;
+    }
+    if (v == -1.0f) *sink = v;
+}
+
+__global__ void mb_empty_kernel() {}
+
+static double time_events(cudaEvent_t a, cudaEvent_t b) {
+    float ms = 0.0f;
+    cudaEventElapsedTime(&ms, a, b);
+    return ms * 1e-3;
+}
+
+int run_microbench(int which, int kind, int ndims, const int64_t* dims, int64_t T, stencil_tile tile,
+                   int threads, double* value) {
+    int dev = 0, nsm = 148;
+    if (cudaGetDevice(&dev) != cudaSuccess) return STENCIL_ENODEV;
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    cudaStream_t s;
+    cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking);
+    cudaEvent_t e0, e1;
+    cudaEventCreate(&e0);
+    cudaEventCreate(&e1);
+    int rc = STENCIL_OK;
+    double best = 1e30;
+    if (which == 0) {
+        const int64_t n = (int64_t)1 << 28;   // 1 GiB per buffer, well above the 126 MB L2
+        float *a = nullptr, *b = nullptr;
+        if (cudaMalloc(&a, n * 4) != cudaSuccess || cudaMalloc(&b, n * 4) != cudaSuccess) {
+            rc = STENCIL_ENOMEM;
+        } else {
+            cudaMemsetAsync(a, 0, n * 4, s);
+            for (int r = 0; r < 12; ++r) {
+                cudaEventRecord(e0, s);
+                mb_copy_kernel<<<nsm * 8, 512, 0, s>>>((const float4*)a, (float4*)b, n / 4);
+                cudaEventRecord(e1, s);
+                cudaEventSynchronize(e1);
+                if (r >= 2) best = std::min(best, time_events(e0, e1));
+            }
+            *value = best / (2.0 * (double)n);       // read + write words
+        }
+        if (a) cudaFree(a);
+        if (b) cudaFree(b);
+    } else if (which == 1) {
+        const int thr = threads > 0 ? threads : 256;
+        const int iters = 1 << 16;
+        float* sink;
+        cudaMalloc(&sink, 4);
+        for (int r = 0; r < 5; ++r) {
+            cudaEventRecord(e0, s);
+            mb_sync_kernel<<<nsm, thr, 0, s>>>(iters, sink);
+            cudaEventRecord(e1, s);
+            cudaEventSynchronize(e1);
+            if (r >= 1) best = std::min(best, time_events(e0, e1));
+        }
+        *value = best / iters;
+        cudaFree(sink);
+    } else if (which == 2) {
+        const int n = 1000;
+        cudaGraph_t g;
+        cudaGraphExec_t ge;
+        cudaStreamBeginCapture(s, cudaStreamCaptureModeThreadLocal);
+        for (int i = 0; i < n; ++i) mb_empty_kernel<<<nsm, 128, 0, s>>>();
+        cudaStreamEndCapture(s, &g);
+        cudaGraphInstantiate(&ge, g, 0);
+        for (int r = 0; r < 6; ++r) {
+            cudaEventRecord(e0, s);
+            cudaGraphLaunch(ge, s);
+            cudaEventRecord(e1, s);
+            cudaEventSynchronize(e1);
+            if (r >= 1) best = std::min(best, time_events(e0, e1));
+        }
+        *value = best / n;
+        cudaGraphExecDestroy(ge);
+        cudaGraphDestroy(g);
+    } else if (which == 3) {
+        // compute-only HHC run, then divide by the EXACT iteration count
+        stencil_t h = nullptr;
+        rc = stencil_create((stencil_kind)kind, ndims, dims, nullptr, 0, STENCIL_MODE_FUSED, &h);
+        if (rc == STENCIL_OK) {
+            const int64_t n = dims[0] * dims[1] * (ndims == 3 ? dims[2] : 1);
+            float *a = nullptr, *b = nullptr;
+            if (cudaMalloc(&a, n * 4) != cudaSuccess || cudaMalloc(&b, n * 4) != cudaSuccess) rc = STENCIL_ENOMEM;
+            if (rc == STENCIL_OK) {
+                cudaMemsetAsync(a, 0, n * 4, s);
+                set_compute_only(h, 1);
+                for (int r = 0; r < 4 && rc == STENCIL_OK; ++r) {
+                    cudaEventRecord(e0, s);
+                    rc = stencil_run(h, a, b, T, tile, threads, s);
+                    cudaEventRecord(e1, s);
+                    cudaEventSynchronize(e1);
+                    if (r >= 1) best = std::min(best, time_events(e0, e1));
+                }
+                set_compute_only(h, 0);
+                model_hw_params hw{};
+                hw.n_sm = nsm; hw.n_v = 128; hw.mtb_sm = 32; hw.r_sm = 65536;
+                int smopt = 0;
+                cudaDeviceGetAttribute(&smopt, cudaDevAttrMaxSharedMemoryPerMultiprocessor, dev);
+                hw.m_sm_bytes = smopt;
+                cudaDeviceGetAttribute(&smopt, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+                hw.m_block_bytes = smopt;
+                hw.L_s_per_word = 0; hw.tau_sync_s = 0; hw.T_sync_s = 0; hw.C_iter_s = 1.0;
+                hw.geometry = 1;
+                hw.threads = threads;
+                const double iters = model_predict((stencil_kind)kind, ndims, dims, T, tile, &hw);
+                *value = best / iters;
+            }
+            if (a) cudaFree(a);
+            if (b) cudaFree(b);
+            stencil_destroy(h);
+        }
+    } else {
+        rc = STENCIL_EINVAL;
+    }
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    cudaStreamDestroy(s);
+    if (rc == STENCIL_OK && cudaGetLastError() != cudaSuccess) rc = STENCIL_ECUDA;
+    return rc;
+}
+
+}  // namespace hhc

@@ -1,0 +1,231 @@
+// model.cpp -- the paper's analytical execution-time model (§4,
+// Eqs. 2-30) and the tile-size optimisation of §6.1 (Eq. 31,
+// P:L1365-1453), host fp64.  Two geometries (reading M1):
+//   PAPER -- the printed equations (readings M2-M5 for the garbled ones);
+//   EXACT -- the same equations on the hexagon and footprints the kernels
+//            implement (readings G1-G3), with Eq. 2's per-row sum.
+// Multi-GPU term (n_gpus > 1): DESIGN.md reading M7.
+#include <algorithm>
+#include <cmath>
+#include <cstdint>
+#include <limits>
+#include <vector>
+
+#include "hhc_internal.h"
+
+namespace {
+
+inline int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
+
+int ndims_of(int kind) {
+    switch (kind) {
+    case STENCIL_JACOBI2D_5PT: case STENCIL_HEAT2D_9PT: case STENCIL_GRADIENT2D:
+    case STENCIL_LAPLACIAN2D_5PT: return 2;
+    case STENCIL_HEAT3D_7PT: case STENCIL_LAPLACIAN3D_27PT: return 3;
+    default: return 0;
+    }
+}
+
+bool tile_ok(int nd, const stencil_tile& t) {
+    if (t.t < 2 || (t.t & 1) || t.s1 < 1 || t.s2 < 1) return false;
+    if (nd == 2) return t.s2 % 32 == 0;
+    return t.s3 >= 32 && t.s3 % 32 == 0;
+}
+
+// ---------------------------------------------------------------- PAPER
+double talg_paper(int nd, const int64_t* S, int64_t T, const stencil_tile& tl, const model_hw_params& hw) {
+    const int64_t tT = tl.t, tS1 = tl.s1, tS2 = tl.s2, tS3 = nd == 3 ? tl.s3 : 1;
+    const int64_t S1 = S[0], S2 = S[1], S3 = nd == 3 ? S[2] : 1;
+    // Eq. 3: Nw = 2 ceil(T/tT) + eps, eps = 0 iff 0 < T - floor(T/tT) tT <= tT/2
+    const int64_t r = T - (T / tT) * tT;
+    const int64_t Nw = 2 * cdiv(T, tT) + ((r > 0 && 2 * r <= tT) ? 0 : 1);
+    const int64_t wtile = tS1 + tT - 2;                        // Eq. 4 / 21
+    const int64_t w = cdiv(S1, 2 * tS1 + tT);                 // Eq. 5 / 22 (reading M2)
+    const int64_t inner = nd == 2 ? tS2 : tS2 * tS3;
+    const double mi = (double)inner * (double)(tS1 + 2 * tT);  // Eq. 13 / 24
+    const double mo = mi;
+    const double m_prime = (mi + mo) * hw.L_s_per_word + 2.0 * hw.tau_sync_s;   // Eq. 14 / 25
+    double sum = 0.0;                                          // Eq. 15 / 27
+    for (int64_t x = tS1; x <= wtile; x += 2) sum += (double)cdiv(x * inner, hw.n_v);
+    const double c = 2.0 * hw.C_iter_s * sum + (double)tT * hw.tau_sync_s;
+    int64_t Mtile;                                             // Eq. 19, reading M3 in 3D (words)
+    double Nsub;
+    if (nd == 2) {
+        Mtile = 2 * (tS1 + tT + 1) * (tS2 + tT + 1);
+        Nsub = (double)cdiv(S2 + tT, tS2);                     // Eq. 16
+    } else {
+        Mtile = 2 * (tS1 + tT + 1) * (tS2 + tT + 1) * (tS3 + tT + 1);
+        Nsub = std::ceil(((double)(S2 + tT) / (double)tS2) * ((double)(S3 + tT) / (double)tS3));   // Eq. 23
+    }
+    const int64_t Mbytes = 4 * Mtile;
+    if (Mbytes > hw.m_block_bytes) return std::numeric_limits<double>::infinity();   // Eq. 31
+    int64_t k = std::min<int64_t>(hw.m_sm_bytes / Mbytes, hw.mtb_sm);               // Eq. 11 (reading M4)
+    if (k < 1) return std::numeric_limits<double>::infinity();
+    double Tprism;
+    if (k == 1) Tprism = (m_prime + c) * Nsub;                                     // Eq. 16 / 28
+    else Tprism = m_prime + (double)k * std::max(m_prime, c) * Nsub;               // Eq. 16 / 29
+    const double rounds = (double)cdiv(cdiv(w, k), hw.n_sm);
+    return (double)Nw * hw.T_sync_s + (double)Nw * Tprism * rounds;                // Eq. 17 / 30
+}
+
+// ---------------------------------------------------------------- EXACT
+inline int64_t row_width(int64_t tau, int64_t tS1, int64_t tT) { return tS1 + 2 * std::min(tau, tT - tau); }
+
+int default_threads(int nd, const stencil_tile& t) {
+    const int base = hhc::column_threads(nd, t.s2, t.s3);
+    const int G = base <= 256 ? std::max(1, std::min(4, 256 / base)) : 1;
+    return base * G;
+}
+
+double talg_exact(int nd, const int64_t* S, int64_t T, const stencil_tile& tl, const model_hw_params& hw) {
+    const int64_t tT = tl.t, tS1 = tl.s1, tS2 = tl.s2, tS3 = nd == 3 ? tl.s3 : 1;
+    const int64_t S1 = S[0], S2 = S[1], S3 = nd == 3 ? S[2] : 1;
+    const int64_t Mtile = hhc::smem_bytes(nd, (int)tT, (int)tS1, (int)tS2, (int)tS3);
+    const int threads = hw.threads > 0 ? hw.threads : default_threads(nd, tl);
+    const int64_t maxthr = hw.max_threads_sm > 0 ? hw.max_threads_sm : 2048;
+    if (Mtile > hw.m_block_bytes || threads > 512) return std::numeric_limits<double>::infinity();
+    int64_t k = std::min<int64_t>({hw.m_sm_bytes / Mtile, (int64_t)hw.mtb_sm, maxthr / threads});   // Eq. 11
+    if (hw.regs_per_thread > 0) k = std::min<int64_t>(k, hw.r_sm / ((int64_t)hw.regs_per_thread * threads));
+    if (k < 1) return std::numeric_limits<double>::infinity();
+    const int64_t P = 2 * tS1 + tT, h = tT / 2;
+    const int64_t wA = cdiv(S1 + h, P);                        // reading G2
+    const int64_t wB = S1 > tS1 ? cdiv(S1 - tS1, P) : 0;
+    const double L_sm = hw.L_s_per_word * hw.n_sm;             // reading M5
+    const int64_t Nw = cdiv(2 * T, tT) + 1;
+    double total = 0.0;
+    // rows with identical (phase, lo, hi, final-level) cost the same: memoise
+    int64_t key_prev[2] = {-1, -1};
+    double val_prev[2] = {0.0, 0.0};
+    for (int64_t m = -1; m <= Nw - 2; ++m) {
+        const int64_t t0 = 1 + m * h;
+        const int64_t lo = std::max<int64_t>(0, 1 - t0);
+        const int64_t hi = std::min<int64_t>(tT, T - t0 + 1);
+        const int64_t nlev = hi - lo;
+        const int ph = (int)(((m % 2) + 2) % 2);
+        const int64_t w = ph == 0 ? wA : wB;
+        total += hw.T_sync_s;
+        if (w == 0 || nlev <= 0) continue;
+        const int64_t fin = (t0 + hi - 1 == T) ? hi - 1 : -1;
+        const int64_t key = ((lo * 4096 + hi) * 4096 + (fin + 1));
+        if (key == key_prev[ph]) { total += val_prev[ph]; continue; }
+        // footprint (reads) and facets (writes) per unit inner extent, reading G3
+        int64_t reads = 0, writes = 0, area = 0;
+        double csum = 0.0;
+        const int64_t inner = nd == 2 ? tS2 : tS2 * tS3;
+        for (int64_t tau = lo; tau < hi; ++tau) {
+            const int64_t W = row_width(tau, tS1, tT);
+            area += W;
+            if (tau == lo) reads += W + 2;
+            else if (tau <= h) reads += 4;
+            if (t0 + tau == T || tau == hi - 1) writes += W;
+            else if (tau + 1 > h) writes += 4;
+            csum += (double)cdiv(W * inner, hw.n_v);           // Eq. 15 / 27, row by row
+        }
+        double Nsub, mi, mo, extra = 0.0;
+        if (nd == 2) {
+            Nsub = (double)cdiv(S2 + nlev - 1, tS2);
+            mi = (double)reads * (double)(tS2 + 2);
+            mo = (double)writes * (double)tS2;
+        } else {
+            Nsub = (double)(cdiv(S2 + nlev - 1, tS2) * cdiv(S3 + nlev - 1, tS3));
+            mi = (double)reads * (double)((tS2 + 2) * (tS3 + 2));
+            mo = (double)writes * (double)(tS2 * tS3);
+            extra = 4.0 * (double)tS3 * (double)area;           // S2 face through global memory
+        }
+        const double m_prime = (mi + mo + extra) * L_sm + 2.0 * hw.tau_sync_s;     // Eq. 14 / 25
+        const double c = csum * hw.C_iter_s + (double)nlev * hw.tau_sync_s;
+        double Tprism;
+        if (k == 1) Tprism = (m_prime + c) * Nsub;                                 // Eq. 16 / 28
+        else Tprism = m_prime + (double)k * std::max(m_prime, c) * Nsub;           // Eq. 16 / 29
+        const double v = Tprism * (double)cdiv(cdiv(w, k), hw.n_sm);              // Eq. 2
+        key_prev[ph] = key;
+        val_prev[ph] = v;
+        total += v;
+    }
+    return total;
+}
+
+// Reading M7 (multi-GPU, not in the paper): G slabs of own = ceil(S1/G) rows,
+// each time tile of tT steps runs HHC on own + 2 tT rows and exchanges tT rows
+// per neighbour: T_G = ceil(T/tT) * (Talg(own + 2 tT, tT) + T_exch).
+double talg_dist(int nd, const int64_t* S, int64_t T, const stencil_tile& tl, const model_hw_params& hw,
+                 double (*f)(int, const int64_t*, int64_t, const stencil_tile&, const model_hw_params&)) {
+    const int64_t G = hw.n_gpus;
+    const int64_t own = cdiv(S[0], G);
+    int64_t Sl[3] = {own + 2 * tl.t, S[1], nd == 3 ? S[2] : 1};
+    const int64_t ntile = cdiv(T, tl.t);
+    double tile_time = f(nd, Sl, tl.t, tl, hw);
+    if (!std::isfinite(tile_time)) return tile_time;
+    const double plane = (double)S[1] * (double)(nd == 3 ? S[2] : 1) * 4.0;
+    const double msg = (double)tl.t * plane;
+    const double bw = hw.link_bytes_per_s > 0 ? hw.link_bytes_per_s : 7.7e11;
+    const double t_exch = msg / bw + hw.link_latency_s;
+    return (double)ntile * (tile_time + t_exch);
+}
+
+}  // namespace
+
+extern "C" double model_predict(stencil_kind kind, int ndims, const int64_t* dims, int64_t T, stencil_tile tile,
+                                const model_hw_params* hw) {
+    const double nan = std::numeric_limits<double>::quiet_NaN();
+    if (!hw || !dims || ndims != ndims_of(kind) || T < 1) return nan;
+    for (int d = 0; d < ndims; ++d)
+        if (dims[d] < 3) return nan;
+    if (!tile_ok(ndims, tile)) return nan;
+    if (hw->n_sm < 1 || hw->n_v < 1 || hw->mtb_sm < 1 || hw->m_sm_bytes < 1 || hw->m_block_bytes < 1) return nan;
+    int64_t S[3] = {dims[0] - 2, dims[1] - 2, ndims == 3 ? dims[2] - 2 : 1};
+    auto f = hw->geometry == 1 ? talg_exact : talg_paper;
+    if (hw->n_gpus > 1) return talg_dist(ndims, S, T, tile, *hw, f);
+    return f(ndims, S, T, tile, *hw);
+}
+
+extern "C" int model_select_tile(stencil_kind kind, int ndims, const int64_t* dims, int64_t T,
+                                 const model_hw_params* hw, double within, stencil_tile* best, int* best_threads,
+                                 stencil_tile* cands, int cap, int* n_cands) {
+    if (!hw || !dims || !best || ndims != ndims_of(kind) || T < 1 || within < 0) return STENCIL_EINVAL;
+    for (int d = 0; d < ndims; ++d)
+        if (dims[d] < 3) return STENCIL_EINVAL;
+    // search space, reading M6
+    const int64_t S1 = dims[0] - 2, S2 = dims[1] - 2, S3 = ndims == 3 ? dims[2] - 2 : 1;
+    const int64_t Tev = T + (T & 1);
+    const int64_t tTmax = std::min<int64_t>(Tev, 128), tS1max = std::min<int64_t>(S1, 64);
+    const int64_t innerS = ndims == 2 ? S2 : S3;
+    const int64_t innermax = std::min<int64_t>(1024, cdiv(innerS, 32) * 32);
+    const int64_t tS2max3 = std::min<int64_t>(S2, 16);
+    struct V { stencil_tile t; double v; };
+    std::vector<V> vals;
+    stencil_tile bt{0, 0, 0, 0};
+    double bv = std::numeric_limits<double>::infinity();
+    for (int64_t tT = 2; tT <= tTmax; tT += 2)
+        for (int64_t tS1 = 1; tS1 <= tS1max; ++tS1) {
+            const int64_t n2 = ndims == 2 ? 1 : tS2max3;
+            for (int64_t a = 1; a <= n2; ++a)
+                for (int64_t in = 32; in <= innermax; in += 32) {
+                    stencil_tile t;
+                    t.t = (int)tT; t.s1 = (int)tS1;
+                    if (ndims == 2) { t.s2 = (int)in; t.s3 = 0; }
+                    else { t.s2 = (int)a; t.s3 = (int)in; }
+                    const double v = model_predict(kind, ndims, dims, T, t, hw);
+                    if (!std::isfinite(v)) {
+                        if (ndims == 2 || true) {
+                            // larger inner tiles only grow Mtile: stop this inner sweep
+                            if (std::isinf(v)) break;
+                        }
+                        continue;
+                    }
+                    vals.push_back(V{t, v});
+                    if (v < bv) { bv = v; bt = t; }   // strict: first (lexicographic) minimum wins
+                }
+        }
+    if (!std::isfinite(bv)) return STENCIL_ETILE;
+    *best = bt;
+    if (best_threads) *best_threads = default_threads(ndims, bt);
+    int n = 0;
+    for (auto& x : vals)
+        if (x.v <= (1.0 + within) * bv) {
+            if (cands && n < cap) cands[n] = x.t;
+            ++n;
+        }
+    if (n_cands) *n_cands = n;
+    return STENCIL_OK;
+}

@@ -1,0 +1,155 @@
+"""CPU-side checks of the C ABI (include/hhc.h / libhhc.so): the library
+loads, exports every declared symbol, rejects bad arguments, and its host
+parts (planner, model_predict, model_select_tile) agree with the oracle.
+No GPU needed (no stencil compute is called here)."""
+import math
+import random
+import re
+import os
+
+import pytest
+
+import paper_conf_ppopp_prajapatirradg17_b200 as hhc
+from oracle import hex_geometry as hg
+from oracle import model_oracle as mo
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module")
+def lib():
+    from paper_conf_ppopp_prajapatirradg17_b200._build import build
+    build()
+    return hhc.load()
+
+
+def header_functions():
+    src = open(os.path.join(ROOT, "include", "hhc.h")).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    names = re.findall(r"^\s*(?:const\s+)?[a-z_0-9]+\*?\s+\**([a-z_0-9]+)\s*\(", src, flags=re.M)
+    return sorted(set(names))
+
+
+def test_exports_every_declared_symbol(lib):
+    names = header_functions()
+    assert len(names) >= 12, names
+    for n in names:
+        assert hasattr(lib, n), n
+    assert set(hhc.EXPORTED_SYMBOLS) == set(names)
+
+
+def test_strerror(lib):
+    assert hhc.strerror(0) == "ok"
+    assert "tile" in hhc.strerror(hhc.ETILE)
+
+
+def test_create_without_gpu_fails_loudly(lib):
+    import torch
+    if torch.cuda.is_available():
+        pytest.skip("GPU present")
+    with pytest.raises(hhc.StencilError) as e:
+        hhc.stencil_create(hhc.HEAT2D_9PT, (64, 64))
+    assert e.value.status in (hhc.ENODEV, hhc.ECUDA)
+
+
+def test_tile_validation(lib):
+    assert hhc.stencil_tile_resources(2, (8, 8, 64))[1] == 64        # 16 column threads x 4 groups
+    for bad in [(7, 8, 64), (0, 8, 64), (8, 0, 64), (8, 8, 48), (8, 8, 0)]:
+        with pytest.raises(hhc.StencilError):
+            hhc.stencil_tile_resources(2, bad)
+    with pytest.raises(hhc.StencilError):
+        hhc.stencil_tile_resources(3, (8, 4, 4, 48))
+    with pytest.raises(hhc.StencilError):                              # smem > 227 KB
+        hhc.stencil_tile_resources(2, (64, 64, 1024))
+    with pytest.raises(hhc.StencilError):                              # threads not a multiple
+        hhc.stencil_tile_resources(2, (8, 8, 64), threads=24)
+    sm, thr = hhc.stencil_tile_resources(3, (8, 4, 4, 32))
+    assert sm == mo.smem_bytes_exact(3, (8, 4, 4, 32)) and thr == mo.default_threads(3, (8, 4, 4, 32))
+
+
+def test_plan_info_matches_tiling(lib):
+    """Nw and the per-row hexagon counts of the planner vs the brute-force tiling."""
+    for tT in (2, 4, 6, 8):
+        for tS in (1, 2, 5):
+            S1, T = 33, 2 * tT + 3
+            rows, w, *_ = hg.analyse(S1, T, tS, tT)
+            nrows, wa, wb, _ = hhc.stencil_plan_info((S1 + 2, 40), T, (tT, tS, 32))
+            assert nrows == len(rows)
+            for m in rows[1:-1]:
+                assert w[m] == (wa if m % 2 == 0 else wb)
+
+
+def hw_pair(kind, geometry, rnd=None, b200=False):
+    o = mo.gtx980(kind, geometry)
+    if b200:
+        o.nSM, o.MSM, o.Mblock = 148, 228 * 1024, 227 * 1024
+    if rnd is not None:
+        o.L *= rnd.uniform(0.2, 5)
+        o.C_iter *= rnd.uniform(0.2, 5)
+        o.tau_sync *= rnd.uniform(0.2, 5)
+        o.regs_per_thread = rnd.choice([0, 0, 40, 64])
+    c = hhc.make_hw(n_sm=o.nSM, n_v=o.nV, mtb_sm=o.MTBSM, r_sm=o.RSM, m_sm_bytes=o.MSM,
+                    m_block_bytes=o.Mblock, L_s_per_word=o.L, tau_sync_s=o.tau_sync, T_sync_s=o.T_sync,
+                    C_iter_s=o.C_iter, regs_per_thread=o.regs_per_thread, geometry=geometry)
+    return o, c
+
+
+def test_model_predict_matches_oracle_hand_example(lib):
+    o, c = hw_pair(3, hhc.PAPER)
+    t = hhc.model_predict(hhc.GRADIENT2D, (8194, 8194), 8192, (8, 8, 256), c)
+    assert abs(t - mo.talg(2, (8192, 8192), 8192, (8, 8, 256, 0), o)) <= 1e-12 * t
+    assert abs(t - 15.96397) < 2e-5
+
+
+@pytest.mark.parametrize("geometry", [hhc.PAPER, hhc.EXACT])
+def test_model_predict_matches_oracle_random(lib, geometry):
+    rnd = random.Random(geometry + 7)
+    n = 0
+    for _ in range(400):
+        kind = rnd.choice([1, 2, 3, 4, 5, 6])
+        nd = hhc.KIND_NDIMS[kind]
+        o, c = hw_pair(kind, geometry, rnd, b200=rnd.random() < 0.5)
+        if nd == 2:
+            S = (rnd.randint(1, 3000), rnd.randint(1, 3000))
+            tile = (2 * rnd.randint(1, 20), rnd.randint(1, 40), 32 * rnd.randint(1, 12), 0)
+        else:
+            S = (rnd.randint(1, 300), rnd.randint(1, 300), rnd.randint(1, 300))
+            tile = (2 * rnd.randint(1, 10), rnd.randint(1, 12), rnd.randint(1, 8), 32 * rnd.randint(1, 4))
+        T = rnd.randint(1, 500)
+        dims = tuple(s + 2 for s in S)
+        got = hhc.model_predict(kind, dims, T, tile, c)
+        exp = mo.talg(nd, S, T, tile, o)
+        if math.isinf(exp):
+            assert math.isinf(got)
+        else:
+            n += 1
+            assert abs(got - exp) <= 1e-12 * exp, (kind, S, T, tile, got, exp)
+    assert n > 100
+
+
+def test_model_predict_invalid_and_infeasible(lib):
+    _, c = hw_pair(2, hhc.PAPER)
+    assert math.isnan(hhc.model_predict(hhc.HEAT2D_9PT, (64, 64), 10, (7, 4, 32), c))
+    assert math.isnan(hhc.model_predict(hhc.HEAT2D_9PT, (64, 64, 64), 10, (8, 4, 32), c))
+    assert math.isnan(hhc.model_predict(hhc.HEAT2D_9PT, (64, 64), 0, (8, 4, 32), c))
+    assert math.isinf(hhc.model_predict(hhc.HEAT2D_9PT, (4098, 4098), 64, (16, 64, 1024), c))
+
+
+@pytest.mark.parametrize("geometry", [hhc.PAPER, hhc.EXACT])
+@pytest.mark.parametrize("kind,S,T", [(2, (60, 70), 12), (3, (45, 100), 9), (4, (20, 18, 40), 6),
+                                      (1, (130, 33), 5)])
+def test_select_tile_matches_oracle(lib, geometry, kind, S, T):
+    o, c = hw_pair(kind, geometry, b200=True)
+    nd = hhc.KIND_NDIMS[kind]
+    best, thr, cands = hhc.model_select_tile(kind, tuple(s + 2 for s in S), T, c, 0.10)
+    ob, ot, oc = mo.select_tile(nd, S, T, o, 0.10)
+    assert best == ob
+    assert cands == oc
+    assert thr == mo.default_threads(nd, best)
+
+
+def test_select_tile_infeasible(lib):
+    _, c = hw_pair(2, hhc.PAPER)
+    c.m_block_bytes = 16
+    with pytest.raises(hhc.StencilError):
+        hhc.model_select_tile(hhc.HEAT2D_9PT, (66, 66), 10, c)

@@ -1,0 +1,219 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle,
+element by element on the same seeded inputs.  Bar (BASELINE.json north_star,
+DESIGN.md R4/R5): bit-exact in both arithmetic modes (plain vs plain oracle,
+fused vs fused oracle); fused within 1e-5 max relative error of the plain
+oracle.  At the full config sizes: exact corner windows (dependence-cone
+argument) plus closed-form / invariant checks over the whole grid."""
+import math
+import os
+
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+import oracle  # noqa: E402
+import paper_conf_ppopp_prajapatirradg17_b200 as hhc  # noqa: E402
+from synth import field  # noqa: E402
+
+if not torch.cuda.is_available():
+    pytest.skip("needs a CUDA device", allow_module_level=True)
+
+DEV = torch.device("cuda:0")
+
+
+def gpu_run(kind, a, T, tile, mode=hhc.FUSED, threads=0, coeffs=None, env=None):
+    old = {}
+    for k, v in (env or {}).items():
+        old[k] = os.environ.get(k)
+        os.environ[k] = v
+    try:
+        s = hhc.stencil_create(kind, a.shape, coeffs=coeffs, mode=mode)
+        d_in = torch.from_numpy(np.ascontiguousarray(a)).to(DEV)
+        d_out = torch.empty_like(d_in)
+        hhc.stencil_run(s, d_in, d_out, T, tile, threads)
+        torch.cuda.synchronize()
+        assert hhc.stencil_last_launches(s) >= 1
+        res = d_out.cpu().numpy()
+        hhc.stencil_destroy(s)
+        return res
+    finally:
+        for k, v in old.items():
+            if v is None:
+                os.environ.pop(k, None)
+            else:
+                os.environ[k] = v
+
+
+def assert_bits(got, exp, what=""):
+    if not np.array_equal(got.view(np.uint32), exp.view(np.uint32)):
+        bad = np.argwhere(got.view(np.uint32) != exp.view(np.uint32))
+        i = tuple(bad[0])
+        raise AssertionError(f"{what}: {len(bad)} mismatches, first at {i}: gpu {got[i]!r} oracle {exp[i]!r}")
+
+
+def max_rel(got, ref):
+    g, r = got.astype(np.float64), ref.astype(np.float64)
+    return float(np.max(np.abs(g - r) / np.maximum(np.abs(r), 2.0 ** -10)))
+
+
+TILES_2D = [(2, 1, 32), (4, 3, 32), (8, 5, 64), (6, 2, 32), (10, 7, 96), (16, 4, 128), (2, 9, 64)]
+TILES_3D = [(2, 1, 1, 32), (4, 2, 3, 32), (6, 3, 4, 64), (8, 2, 2, 32), (2, 5, 6, 32)]
+
+
+@pytest.mark.parametrize("kind", [hhc.JACOBI2D_5PT, hhc.HEAT2D_9PT, hhc.GRADIENT2D, hhc.LAPLACIAN2D_5PT])
+@pytest.mark.parametrize("mode", [hhc.PLAIN, hhc.FUSED])
+def test_parity_2d_small(kind, mode):
+    rng = np.random.default_rng(kind * 10 + mode)
+    for tile in TILES_2D:
+        dims = (int(rng.integers(3, 90)), int(rng.integers(3, 150)))
+        a = field(int(rng.integers(1, 1 << 30)), dims)
+        for T in (1, 2, 5, tile[0] + 1, 2 * tile[0] + 3):
+            got = gpu_run(kind, a, T, tile, mode)
+            exp = oracle.run(kind, a, T, mode)
+            assert_bits(got, exp, f"kind {kind} mode {mode} dims {dims} T {T} tile {tile}")
+
+
+@pytest.mark.parametrize("kind", [hhc.HEAT3D_7PT, hhc.LAPLACIAN3D_27PT])
+@pytest.mark.parametrize("mode", [hhc.PLAIN, hhc.FUSED])
+def test_parity_3d_small(kind, mode):
+    rng = np.random.default_rng(kind * 10 + mode)
+    for tile in TILES_3D:
+        dims = (int(rng.integers(3, 30)), int(rng.integers(3, 30)), int(rng.integers(3, 80)))
+        a = field(int(rng.integers(1, 1 << 30)), dims)
+        for T in (1, 3, tile[0] + 1, 2 * tile[0] + 1):
+            exp = oracle.run(kind, a, T, mode)
+            got = gpu_run(kind, a, T, tile, mode)
+            assert_bits(got, exp, f"kind {kind} dims {dims} T {T} tile {tile}")
+            got1 = gpu_run(kind, a, T, tile, mode, env={"HHC_J": "1"})      # single block per slab
+            assert_bits(got1, exp, f"J=1 kind {kind} dims {dims} T {T} tile {tile}")
+
+
+@pytest.mark.parametrize("threads", [0, 8, 16, 24, 64])
+def test_threads_variants(threads):
+    a = field(5, (77, 133))
+    tile = (6, 3, 32)
+    exp = oracle.run(hhc.HEAT2D_9PT, a, 19, hhc.FUSED)
+    got = gpu_run(hhc.HEAT2D_9PT, a, 19, tile, hhc.FUSED, threads=threads)
+    assert_bits(got, exp, f"threads {threads}")
+
+
+def test_T0_and_tiny_grids():
+    a = field(3, (3, 3))
+    assert_bits(gpu_run(hhc.HEAT2D_9PT, a, 0, (2, 1, 32)), a)
+    assert_bits(gpu_run(hhc.HEAT2D_9PT, a, 4, (2, 1, 32)), oracle.run(hhc.HEAT2D_9PT, a, 4, hhc.FUSED))
+    b = field(4, (3, 3, 3))
+    assert_bits(gpu_run(hhc.LAPLACIAN3D_27PT, b, 3, (2, 1, 1, 32)),
+                oracle.run(hhc.LAPLACIAN3D_27PT, b, 3, hhc.FUSED))
+    c = field(6, (40, 5))        # tile far larger than the grid
+    assert_bits(gpu_run(hhc.JACOBI2D_5PT, c, 9, (16, 30, 256)), oracle.run(hhc.JACOBI2D_5PT, c, 9, hhc.FUSED))
+
+
+def test_custom_coefficients_and_c():
+    a = field(8, (50, 70))
+    offs, w = oracle.stencil_info(hhc.HEAT2D_9PT)
+    coeffs = [float(x) * 0.9 for x in w] + [0.01]
+    for mode in (hhc.PLAIN, hhc.FUSED):
+        exp = oracle.run(hhc.HEAT2D_9PT, a, 11, mode, coeffs=coeffs)
+        got = gpu_run(hhc.HEAT2D_9PT, a, 11, (4, 3, 32), mode, coeffs=coeffs)
+        assert_bits(got, exp, f"coeffs mode {mode}")
+    exp = oracle.run(hhc.GRADIENT2D, a, 7, hhc.FUSED, coeffs=[0.2])
+    assert_bits(gpu_run(hhc.GRADIENT2D, a, 7, (4, 2, 32), coeffs=[0.2]), exp, "kappa")
+
+
+@pytest.mark.parametrize("kind,dims,T,tile", [
+    (hhc.JACOBI2D_5PT, (256, 256), 64, (8, 8, 64)),                 # C1 exactly
+    (hhc.HEAT2D_9PT, (1030, 1100), 64, (16, 20, 128)),
+    (hhc.GRADIENT2D, (700, 900), 40, (8, 6, 256)),
+    (hhc.HEAT3D_7PT, (64, 66, 130), 20, (8, 4, 4, 32)),
+    (hhc.LAPLACIAN3D_27PT, (60, 50, 70), 12, (4, 3, 4, 64)),
+])
+def test_parity_mid_size(kind, dims, T, tile):
+    a = field(42, dims)
+    for mode in (hhc.PLAIN, hhc.FUSED):
+        exp = oracle.run(kind, a, T, mode)
+        got = gpu_run(kind, a, T, tile, mode)
+        assert_bits(got, exp, f"{kind} {dims} mode {mode}")
+    plain = oracle.run(kind, a, T, hhc.PLAIN)
+    assert max_rel(gpu_run(kind, a, T, tile, hhc.FUSED), plain) <= 1e-5
+
+
+# ---- full BASELINE.json sizes, in the launch configuration bench.py times
+FULL = [
+    ("C1", hhc.JACOBI2D_5PT, (256, 256), 64),
+    ("C2", hhc.HEAT2D_9PT, (8192, 8192), 1024),
+    ("C3", hhc.GRADIENT2D, (16384, 16384), 512),
+    ("C4", hhc.HEAT3D_7PT, (512, 512, 512), 256),
+    ("C5", hhc.LAPLACIAN3D_27PT, (768, 768, 768), 128),
+]
+
+
+def bench_tile(cfg):
+    import bench
+    return bench.CONFIGS[cfg]["tile"]
+
+
+@pytest.mark.parametrize("cfg,kind,dims,T", FULL)
+def test_full_size_corner_windows(cfg, kind, dims, T):
+    """Exact check at the full size: out(T, s) depends only on in within
+    distance T of s, so the oracle on a corner window of side T+6 (its far
+    faces act as a fake ring) is exact on the 4-cell corner block."""
+    from synth import CONFIG_SEEDS
+    a = field(CONFIG_SEEDS[cfg], dims)
+    tile = bench_tile(cfg)
+    got = gpu_run(kind, a, T, tile, hhc.FUSED)
+    K = T + 6
+    nd = len(dims)
+    for corner in range(2 ** nd if nd == 2 else 2):
+        sl_in, sl_cmp = [], []
+        for d in range(nd):
+            hi = (corner >> d) & 1
+            if hi:
+                sl_in.append(slice(dims[d] - K, dims[d]))
+            else:
+                sl_in.append(slice(0, K))
+        sub = np.ascontiguousarray(a[tuple(sl_in)])
+        if min(sub.shape) < K:
+            sub = a
+        ref = oracle.run(kind, sub, T, hhc.FUSED)
+        for d in range(nd):
+            hi = (corner >> d) & 1
+            sl_cmp.append(slice(K - 4, K) if hi else slice(0, 4))
+        g = got[tuple(sl_in)][tuple(sl_cmp)]
+        r = ref[tuple(sl_cmp)]
+        assert_bits(np.ascontiguousarray(g), np.ascontiguousarray(r), f"{cfg} corner {corner}")
+    # global invariant: values stay in [min, max] of the input (positive weights / gradient)
+    assert got.min() >= a.min() - 1e-6 and got.max() <= a.max() + 1e-6
+
+
+@pytest.mark.parametrize("cfg,kind,dims,T", FULL[1:])
+def test_full_size_closed_forms(cfg, kind, dims, T):
+    """Whole-grid checks at full size: affine fields are exact fixed points
+    (dyadic kinds and Gradient), and a sine mode decays by lambda^T."""
+    tile = bench_tile(cfg)
+    nd = len(dims)
+    aff = np.ones(dims, np.float32)
+    for d, c in zip(range(nd), (1.0, 2.0, 3.0)):
+        aff += (c * np.arange(dims[d], dtype=np.float32)).reshape([-1 if e == d else 1 for e in range(nd)])
+    got = gpu_run(kind, aff, T, tile, hhc.FUSED)
+    assert np.array_equal(got, aff), cfg
+    if kind == hhc.GRADIENT2D:
+        return
+    offs, w = oracle.stencil_info(kind)
+    p = (3, 5, 2)[:nd]
+    th = np.array([math.pi * p[d] / (dims[d] - 1) for d in range(nd)])
+    lam = sum(float(wj) * np.prod(np.cos(th * o[:nd])) for o, wj in zip(offs, w))
+    sines = []
+    for d in range(nd):
+        sv = np.sin(th[d] * np.arange(dims[d]))
+        sv[0] = sv[-1] = 0.0
+        sines.append(sv)
+    rest = sines[1][:, None] * sines[2][None, :] if nd == 3 else sines[1]
+    u32 = (sines[0].reshape([-1] + [1] * (nd - 1)) * rest[None]).astype(np.float32)
+    got = gpu_run(kind, u32, T, tile, hhc.FUSED)
+    del u32
+    tol = (4 * T * len(w) + 2) * 2.0 ** -24
+    for x0 in range(0, dims[0], 64):                  # slab-wise, bounded host memory
+        ex = (lam ** T) * sines[0][x0:x0 + 64].reshape([-1] + [1] * (nd - 1)) * rest[None]
+        assert np.max(np.abs(got[x0:x0 + 64].astype(np.float64) - ex)) <= tol, (cfg, lam, x0)
