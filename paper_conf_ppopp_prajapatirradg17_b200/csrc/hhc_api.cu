@@ -77,6 +77,7 @@ struct stencil_s {
     float w[kMaxPts] = {};
     float c = 0.0f, kappa = 0.125f;
     bool has_c = false;
+    bool defw = true;           // default weights -> immediate-operand kernels
     int device = 0, nsm = 148, smem_optin = 227 * 1024;
     float* scratch = nullptr;
     unsigned* flags = nullptr;
@@ -89,6 +90,7 @@ struct stencil_s {
     std::vector<GraphEntry> graphs;
     uint64_t use_clock = 0;
     int compute_only = 0;
+    int occ = 1;
 
     int64_t nelem() const { return dims[0] * dims[1] * dims[2]; }
 };
@@ -137,6 +139,7 @@ extern "C" int stencil_create(stencil_kind kind, int ndims, const int64_t* dims,
         if (coeffs) {
             if (ncoeffs != 1) { delete h; return STENCIL_EINVAL; }
             h->kappa = coeffs[0];
+            h->defw = h->kappa == 0.125f;
         }
     } else {
         int n = 0;
@@ -150,8 +153,11 @@ extern "C" int stencil_create(stencil_kind kind, int ndims, const int64_t* dims,
         h->npts = n;
         if (coeffs) {
             if (ncoeffs != n && ncoeffs != n + 1) { delete h; return STENCIL_EINVAL; }
-            for (int j = 0; j < n; ++j) h->w[j] = coeffs[j];
-            if (ncoeffs == n + 1 && coeffs[n] != 0.0f) { h->has_c = true; h->c = coeffs[n]; }
+            for (int j = 0; j < n; ++j) {
+                if (coeffs[j] != h->w[j] || std::signbit(coeffs[j]) != std::signbit(h->w[j])) h->defw = false;
+                h->w[j] = coeffs[j];
+            }
+            if (ncoeffs == n + 1 && coeffs[n] != 0.0f) { h->has_c = true; h->c = coeffs[n]; h->defw = false; }
         }
     }
     if (cudaStreamCreateWithFlags(&h->cap_stream, cudaStreamNonBlocking) != cudaSuccess) {
@@ -262,6 +268,45 @@ extern "C" int stencil_plan_info(int ndims, const int64_t* dims, int64_t T, sten
     return STENCIL_OK;
 }
 
+static int choose_J(stencil_t h, const RowPlan& r) {
+    const int cap = std::max(1, h->nsm * std::max(h->occ, 1) / std::max(r.w, 1));
+    int J = std::max(1, std::min(r.n2, cap));
+    const char* envJ = getenv("HHC_J");
+    if (envJ) J = std::max(1, std::min({atoi(envJ), r.n2, cap}));
+    return J;
+}
+
+// Everything that must not happen inside stream capture: the kernel's smem
+// attribute, its occupancy (for J), and the 3D flag buffer.
+static int prepare_rows(stencil_t h, const int64_t* dims, int64_t T, stencil_tile tile, int thr) {
+    hex_kernel_t k = get_hex_kernel(h->ndims, h->kind, h->mode, h->has_c, h->defw);
+    if (!k) return STENCIL_EINVAL;
+    const int64_t smem = smem_bytes(h->ndims, tile.t, tile.s1, tile.s2, tile.s3);
+    cudaError_t e = cudaFuncSetAttribute((const void*)k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return cuda_fail(h, e);
+    if (h->ndims != 3) return STENCIL_OK;
+    int occ = 1;
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, (const void*)k, thr, (size_t)smem);
+    if (e != cudaSuccess) return cuda_fail(h, e);
+    h->occ = std::max(occ, 1);
+    std::vector<RowPlan> rows;
+    plan_rows(h->ndims, dims, T, tile, rows);
+    int64_t need = 0;
+    for (auto& r : rows) {
+        const int J = choose_J(h, r);
+        if (J > 1) need = std::max<int64_t>(need, (int64_t)r.w * r.n2);
+    }
+    if (need > h->flags_n) {
+        if (h->flags) cudaFree(h->flags);
+        h->flags = nullptr;
+        h->flags_n = 0;
+        e = cudaMalloc(&h->flags, need * sizeof(unsigned));
+        if (e != cudaSuccess) return cuda_fail(h, e);
+        h->flags_n = need;
+    }
+    return STENCIL_OK;
+}
+
 // Enqueue the hexagon rows (a3) for a domain of extents dims whose level 0 is
 // in plane0 (ring included) and whose ring is also present in plane1; the
 // result (level T) lands in plane[T & 1].  Ring values are read from `ring`.
@@ -270,36 +315,21 @@ static int enqueue_rows(stencil_t h, const int64_t* dims, const float* ring, flo
                         std::vector<cudaEvent_t>* evs = nullptr) {
     std::vector<RowPlan> rows;
     plan_rows(h->ndims, dims, T, tile, rows);
-    hex_kernel_t k = get_hex_kernel(h->ndims, h->kind, h->mode, h->has_c);
+    hex_kernel_t k = get_hex_kernel(h->ndims, h->kind, h->mode, h->has_c, h->defw);
     if (!k) return STENCIL_EINVAL;
     const int64_t smem = smem_bytes(h->ndims, tile.t, tile.s1, tile.s2, tile.s3);
-    cudaError_t e = cudaFuncSetAttribute((const void*)k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return cuda_fail(h, e);
     int64_t nl = 0;
+    cudaError_t e;
     // 3D: thread blocks per slab J (pipelined along S2, flags in global memory);
     // all blocks of a launch must be co-resident when J > 1 (no deadlock).
+    // Occupancy and the flag buffer come from prepare_rows (outside capture).
     if (h->ndims == 3) {
-        int occ = 1;
-        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, (const void*)k, thr, (size_t)smem);
-        if (e != cudaSuccess) return cuda_fail(h, e);
-        occ = std::max(occ, 1);
         int64_t need = 0;
-        const char* envJ = getenv("HHC_J");
         for (auto& r : rows) {
-            const int cap = std::max(1, h->nsm * occ / std::max(r.w, 1));
-            int J = std::max(1, std::min(r.n2, cap));
-            if (envJ) J = std::max(1, std::min({atoi(envJ), r.n2, cap}));
-            r.J = J;
-            if (J > 1) need = std::max<int64_t>(need, (int64_t)r.w * r.n2);
+            r.J = choose_J(h, r);
+            if (r.J > 1) need = std::max<int64_t>(need, (int64_t)r.w * r.n2);
         }
-        if (need > h->flags_n) {
-            if (h->flags) cudaFree(h->flags);
-            h->flags = nullptr;
-            h->flags_n = 0;
-            e = cudaMalloc(&h->flags, need * sizeof(unsigned));
-            if (e != cudaSuccess) return cuda_fail(h, e);
-            h->flags_n = need;
-        }
+        if (need > h->flags_n) return STENCIL_EINVAL;   // prepare_rows was not called
         if (need > 0) {
             e = cudaMemsetAsync(h->flags, 0, need * sizeof(unsigned), s);
             if (e != cudaSuccess) return cuda_fail(h, e);
@@ -372,6 +402,8 @@ static bool same_spec(const RunSpec& x, const RunSpec& y) {
 
 // Run a spec through the CUDA-graph cache (captured once per spec, replayed).
 static int run_spec(stencil_t h, const RunSpec& r, cudaStream_t s) {
+    int prc = prepare_rows(h, r.dims, r.T, r.tile, r.thr);
+    if (prc) return prc;
     const bool use_graph = getenv("HHC_NO_GRAPH") == nullptr && !h->compute_only;
     if (!use_graph) {
         int64_t nl = 0;
@@ -498,6 +530,8 @@ extern "C" int stencil_profile(stencil_t h, const float* d_in, float* d_out, int
     plane[1 - (T & 1)] = h->scratch;
     launch_copy_full(d_in, plane[0], n, s);
     launch_copy_ring(d_in, plane[1], h->dims[0], h->dims[1], h->dims[2], s);
+    rc = prepare_rows(h, h->dims, T, tile, thr);
+    if (rc) return rc;
     std::vector<cudaEvent_t> evs;
     int64_t nl = 0;
     rc = enqueue_rows(h, h->dims, d_in, plane[0], plane[1], T, tile, G, thr, s, &nl, &evs);

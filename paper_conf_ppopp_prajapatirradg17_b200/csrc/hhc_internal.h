@@ -33,11 +33,13 @@ struct HexParams {
 };
 
 // Shared-memory bytes of the HHC kernels (DESIGN.md §Kernels K1/K2): two parity
-// planes in skewed coordinates plus a double-buffered skewed face.
+// planes in skewed coordinates, a double-buffered skewed face and the
+// per-level footprint geometry table.
 inline int64_t smem_bytes(int ndims, int tT, int tS1, int tS2, int tS3) {
     const int64_t NX = tS1 + tT + 2;
-    if (ndims == 2) return 4 * (2 * NX * (tS2 + 4) + 2 * (int64_t)tT * NX * 2);
-    return 4 * (2 * NX * (tS2 + 2) * (tS3 + 4) + 2 * (int64_t)tT * NX * (tS2 + 2) * 2);
+    const int64_t geo = 8 * (int64_t)tT;               // per-level footprint geometry (ints)
+    if (ndims == 2) return 4 * (2 * NX * (tS2 + 4) + 2 * (int64_t)tT * NX * 2 + geo);
+    return 4 * (2 * NX * (tS2 + 2) * (tS3 + 4) + 2 * (int64_t)tT * NX * (tS2 + 2) * 2 + geo);
 }
 
 inline int column_threads(int ndims, int tS2, int tS3) {
@@ -45,8 +47,8 @@ inline int column_threads(int ndims, int tS2, int tS3) {
 }
 
 typedef void (*hex_kernel_t)(HexParams);
-hex_kernel_t get_hex_kernel(int ndims, int kind, int mode, bool has_c);
-int hex_kernel_regs(int ndims, int kind, int mode, bool has_c);
+hex_kernel_t get_hex_kernel(int ndims, int kind, int mode, bool has_c, bool defw);
+int hex_kernel_regs(int ndims, int kind, int mode, bool has_c, bool defw);
 void launch_copy_ring(const float* in, float* out, int64_t S1, int64_t S2, int64_t S3, void* stream);
 void launch_copy_full(const float* in, float* out, int64_t n, void* stream);
 
