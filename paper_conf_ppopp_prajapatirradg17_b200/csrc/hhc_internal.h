@@ -7,7 +7,8 @@
 
 namespace hhc {
 
-constexpr int kColsPerThread = 4;   // B: inner-dimension columns per thread (float4)
+constexpr int kCols2D = 4;          // B: inner-dimension columns per thread, 2D kernel (one float4)
+constexpr int kCols3D = 4;          // B: 3D kernel (one float4)
 constexpr int kMaxPts = 27;
 
 // Kernel parameters for one launch = one row of hexagons.
@@ -37,13 +38,13 @@ struct HexParams {
 // per-level footprint geometry table.
 inline int64_t smem_bytes(int ndims, int tT, int tS1, int tS2, int tS3) {
     const int64_t NX = tS1 + tT + 2;
-    const int64_t geo = 8 * (int64_t)tT;               // per-level footprint geometry (ints)
+    const int64_t geo = 16 * (int64_t)tT;              // per-level geometry table (ints)
     if (ndims == 2) return 4 * (2 * NX * (tS2 + 4) + 2 * (int64_t)tT * NX * 2 + geo);
     return 4 * (2 * NX * (tS2 + 2) * (tS3 + 4) + 2 * (int64_t)tT * NX * (tS2 + 2) * 2 + geo);
 }
 
 inline int column_threads(int ndims, int tS2, int tS3) {
-    return ndims == 2 ? tS2 / kColsPerThread : (tS3 / kColsPerThread) * tS2;
+    return ndims == 2 ? tS2 / kCols2D : (tS3 / kCols3D) * tS2;
 }
 
 typedef void (*hex_kernel_t)(HexParams);
