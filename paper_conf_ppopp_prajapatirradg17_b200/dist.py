@@ -1,0 +1,180 @@
+"""Multi-GPU slab decomposition of the HHC path (BASELINE.json
+north_star -- not in the paper).
+
+The interior S1 rows are split into `world` contiguous slabs of
+own = ceil((S1-2)/world) rows.  Every time tile of tT steps:
+
+  1. ghost exchange: each rank sends its first / last g = tT owned rows to
+     rank -/+ 1 and receives its top / bottom ghost rows (torch.distributed
+     P2P: NCCL over NVLink on GPUs, gloo in the CPU tests);
+  2. the rank runs tT steps of HHC on its ghost-extended slab with the
+     slab's outermost rows held fixed (stencil_run_planes, all compute in the
+     CUDA kernels).  After tT steps every owned row is exact, because the
+     dependence cone of tT steps of a radius-1 stencil reaches tT rows.
+
+The level-0 plane of the next tile is the output plane of this one (tT even),
+so no copy is made between tiles.  All collectives are point to point; there
+is no reduction on the data path.  Orchestration only: the per-tile stepper is
+a callable so the CPU tests can run the same driver with the oracle as stepper.
+"""
+from __future__ import annotations
+
+import math
+import os
+import time
+from dataclasses import dataclass
+
+
+@dataclass
+class Slab:
+    rank: int
+    world: int
+    S1: int
+    own: int        # interior rows per rank (last rank may own fewer)
+    r0: int         # first owned interior row
+    r1: int         # one past the last owned interior row
+    e0: int         # first row of the ghost-extended slab
+    e1: int         # one past the last row of the extended slab
+    g: int          # ghost depth (= tT)
+
+    @property
+    def rows(self) -> int:
+        return self.e1 - self.e0
+
+    @property
+    def held(self):
+        """Rows of the global grid the rank's in/out slab holds: the owned
+        rows plus the physical ring row on the edge ranks."""
+        lo = self.r0 - (1 if self.rank == 0 else 0)
+        hi = self.r1 + (1 if self.rank == self.world - 1 else 0)
+        return lo, hi
+
+
+def partition(S1: int, world: int, rank: int, g: int) -> Slab:
+    interior = S1 - 2
+    own = -(-interior // world)
+    r0 = 1 + rank * own
+    r1 = min(1 + (rank + 1) * own, S1 - 1)
+    if r1 <= r0:
+        raise ValueError(f"rank {rank} owns no rows (S1={S1}, world={world})")
+    if world > 1 and own < g:
+        raise ValueError(f"slab of {own} rows is thinner than the ghost depth {g}: use a smaller tT")
+    if world > 1 and r1 - r0 < g and rank < world - 1:
+        raise ValueError("slab thinner than the ghost depth")
+    e0 = max(0, r0 - g)
+    e1 = min(S1, r1 + g)
+    return Slab(rank, world, S1, own, r0, r1, e0, e1, g)
+
+
+def exchange(slab: Slab, plane, xp_dist):
+    """Fill the ghost rows of `plane` (the extended slab, rows e0..e1) from the
+    neighbours' owned rows.  `xp_dist` is torch.distributed."""
+    import torch
+    ops = []
+    g = slab.g
+    lo = slab.r0 - slab.e0          # local index of the first owned row
+    hi = slab.r1 - slab.e0          # local index one past the last owned row
+    if slab.rank > 0:
+        up_send = plane[lo:lo + g]
+        up_recv = plane[lo - g:lo]
+        ops.append(xp_dist.P2POp(xp_dist.isend, up_send.contiguous(), slab.rank - 1))
+        ops.append(xp_dist.P2POp(xp_dist.irecv, up_recv, slab.rank - 1))
+    if slab.rank < slab.world - 1:
+        dn_send = plane[hi - g:hi]
+        dn_recv = plane[hi:hi + g]
+        ops.append(xp_dist.P2POp(xp_dist.isend, dn_send.contiguous(), slab.rank + 1))
+        ops.append(xp_dist.P2POp(xp_dist.irecv, dn_recv, slab.rank + 1))
+    if ops:
+        for r in xp_dist.batch_isend_irecv(ops):
+            r.wait()
+    return torch
+
+
+def run_slabs(slab: Slab, plane0, plane1, T: int, tT: int, stepper, xp_dist):
+    """Drive the time tiles.  plane0 holds level 0 of the extended slab (ring and
+    ghosts included); stepper(plane0, plane1, Tt) runs Tt steps leaving the
+    result in plane0 (Tt even) or plane1 (Tt odd).  Returns the plane holding A_T."""
+    done = 0
+    cur = plane0
+    while done < T:
+        Tt = min(tT, T - done)
+        if slab.world > 1:
+            exchange(slab, cur, xp_dist)
+        out = stepper(cur, plane1 if cur is plane0 else plane0, Tt)
+        cur = out
+        done += Tt
+    return cur
+
+
+def gpu_stepper(handle, tile, threads, stream=None):
+    import paper_conf_ppopp_prajapatirradg17_b200 as hhc
+
+    def step(p0, p1, Tt):
+        hhc.stencil_run_planes(handle, p0.shape[0], p0, p1, Tt, tile, threads, stream)
+        return p0 if Tt % 2 == 0 else p1
+    return step
+
+
+def bench_main(args, cfg, cfgname, configs):
+    """bench.py under torchrun: strong scaling of the config across ranks."""
+    import json
+
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_ppopp_prajapatirradg17_b200 as hhc
+    from synth import CONFIG_SEEDS, field
+
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", str(args.gpus)))
+    local = int(os.environ.get("LOCAL_RANK", str(rank)))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    dist.init_process_group("nccl", device_id=dev)
+    tile = tuple(int(x) for x in args.tile.split(",")) if args.tile else cfg["tile"]
+    tile = tile + (0,) * (4 - len(tile))
+    threads = cfg["threads"] if args.threads is None else args.threads
+    dims, T, kind = cfg["dims"], cfg["T"], cfg["kind"]
+    tT = tile[0]
+    slab = partition(dims[0], world, rank, tT)
+    ext_dims = (slab.rows,) + tuple(dims[1:])
+    host = field(CONFIG_SEEDS[cfgname], dims, row_start=slab.e0, nrows=slab.rows)
+    init = torch.from_numpy(host).to(dev)
+    p0 = torch.empty_like(init)
+    p1 = torch.empty_like(init)
+    h = hhc.stencil_create(kind, ext_dims, mode=hhc.FUSED if args.mode == "fused" else hhc.PLAIN)
+    stream = torch.cuda.current_stream()
+    step = gpu_stepper(h, tile, threads, stream)
+
+    def one():
+        p0.copy_(init)
+        return run_slabs(slab, p0, p1, T, tT, step, dist)
+
+    for _ in range(args.warmup):
+        one()
+    torch.cuda.synchronize()
+    dist.barrier()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for _ in range(args.steps):
+        one()
+    e1.record(stream)
+    torch.cuda.synchronize()
+    dist.barrier()
+    t = torch.tensor([e0.elapsed_time(e1) * 1e-3], device=dev)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    dt = float(t.item())
+    n_upd = hhc.updates(dims, T)
+    if rank == 0:
+        line = {"metric": "GStencil-updates/s", "value": round(n_upd * args.steps / dt / 1e9, 3),
+                "unit": "GStencil-updates/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+                "ms_per_step": round(dt / args.steps * 1e3, 3), "higher_is_better": True, "scaling": "strong",
+                "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+                "config": {"workload": cfgname + ": " + cfg["desc"], "tile": list(tile), "threads": threads,
+                           "parallelism": f"{world} S1 slabs, ghost depth {tT}, NCCL P2P every time tile",
+                           "l2": "inputs larger than L2"},
+                "gpu_launches": None}
+        print(json.dumps(line))
+    hhc.stencil_destroy(h)
+    dist.destroy_process_group()
+    return 0

@@ -1,0 +1,262 @@
+"""Calibration, validation and tile selection on B200.
+
+    python -m paper_conf_ppopp_prajapatirradg17_b200.tune calibrate [--out profiles/hw_params_b200.json]
+    python -m paper_conf_ppopp_prajapatirradg17_b200.tune sweep  --config C2 [--out ...]
+    python -m paper_conf_ppopp_prajapatirradg17_b200.tune select --config C2
+
+* calibrate -- the micro-benchmarks of PAPER.md §5.2 (L1265-1303): L, tau_sync,
+  T_sync from dedicated kernels; C_iter per stencil from the compute-only HHC
+  kernel over random problem/tile instances (the paper uses 70), averaged.
+* sweep -- measured time of a grid of tiles (minimum of repeated runs)
+  next to Talg (PAPER and EXACT geometry with the calibrated constants); RMSE of
+  (Talg - Texec)/Texec over all points and over points within 20% of the best
+  (reading Q15), and the chosen-tile gaps of reading Q17.
+* select -- Eq. 31 by enumeration (model_select_tile), then measure every tile
+  within 10% of Talg_min and keep the fastest.
+
+All timing is CUDA events on the launching stream; all compute runs in libhhc.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import random
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+if ROOT not in sys.path:
+    sys.path.insert(0, ROOT)
+
+import paper_conf_ppopp_prajapatirradg17_b200 as hhc  # noqa: E402
+
+KINDS = [hhc.JACOBI2D_5PT, hhc.HEAT2D_9PT, hhc.LAPLACIAN2D_5PT, hhc.GRADIENT2D, hhc.HEAT3D_7PT,
+         hhc.LAPLACIAN3D_27PT]
+
+
+def b200_hw(cal: dict | None, kind: int, geometry: int, threads: int = 0) -> "hhc.model_hw_params":
+    """Table 2 analogue for B200 plus calibrated Table 3/4 constants."""
+    import torch
+    props = torch.cuda.get_device_properties(0) if torch.cuda.is_available() else None
+    n_sm = props.multi_processor_count if props else 148
+    hw = hhc.make_hw(n_sm=n_sm, n_v=128, mtb_sm=32, r_sm=65536, m_sm_bytes=228 * 1024,
+                     m_block_bytes=227 * 1024, geometry=geometry, threads=threads, max_threads_sm=2048)
+    if cal:
+        hw.L_s_per_word = cal["L_s_per_word"]
+        hw.tau_sync_s = cal["tau_sync_s"]
+        hw.T_sync_s = cal["T_sync_s"]
+        hw.C_iter_s = cal["C_iter_s"][str(kind)]
+    return hw
+
+
+def load_cal(path=None):
+    path = path or os.path.join(ROOT, "profiles", "hw_params_b200.json")
+    with open(path) as f:
+        return json.load(f)
+
+
+def time_run(h, d_in, d_out, T, tile, threads, reps=3):
+    """min over reps of CUDA-event time of one stencil_run (after one warm run)."""
+    import torch
+    s = torch.cuda.current_stream()
+    hhc.stencil_run(h, d_in, d_out, T, tile, threads, s)
+    torch.cuda.synchronize()
+    best = math.inf
+    for _ in range(reps):
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(s)
+        hhc.stencil_run(h, d_in, d_out, T, tile, threads, s)
+        b.record(s)
+        b.synchronize()
+        best = min(best, a.elapsed_time(b) * 1e-3)
+    return best
+
+
+def random_tile(rnd, nd, dims):
+    if nd == 2:
+        return (2 * rnd.randint(1, 12), rnd.randint(1, 32), 32 * rnd.randint(1, 8), 0)
+    return (2 * rnd.randint(1, 6), rnd.randint(1, 8), rnd.randint(1, 6), 32 * rnd.randint(1, 2))
+
+
+def calibrate(args):
+    out = {"device": None, "how": "PAPER.md §5.2 micro-benchmarks re-measured on this GPU"}
+    import torch
+    out["device"] = torch.cuda.get_device_name(0)
+    out["L_s_per_word"] = hhc.stencil_microbench(0)
+    out["L_s_per_GB"] = out["L_s_per_word"] / 4e-9
+    out["tau_sync_s"] = hhc.stencil_microbench(1, threads=256)
+    out["T_sync_s"] = hhc.stencil_microbench(2)
+    rnd = random.Random(2017)
+    citer, samples = {}, {}
+    for kind in KINDS:
+        nd = hhc.KIND_NDIMS[kind]
+        vals = []
+        while len(vals) < args.instances:
+            if nd == 2:
+                dims = (rnd.randint(1024, 4096), rnd.randint(1024, 4096))
+                T = rnd.randint(16, 64)
+            else:
+                dims = (rnd.randint(96, 256), rnd.randint(96, 256), rnd.randint(96, 256))
+                T = rnd.randint(8, 24)
+            tile = random_tile(rnd, nd, dims)
+            try:
+                hhc.stencil_tile_resources(nd, tile)
+            except hhc.StencilError:
+                continue
+            v = hhc.stencil_microbench(3, kind, dims, T, tile)
+            if math.isfinite(v) and v > 0:
+                vals.append(v)
+        citer[str(kind)] = sum(vals) / len(vals)
+        samples[str(kind)] = {"n": len(vals), "min": min(vals), "max": max(vals)}
+        print(f"C_iter kind {kind}: {citer[str(kind)]:.3e} s over {len(vals)} instances", flush=True)
+    out["C_iter_s"] = citer
+    out["C_iter_samples"] = samples
+    os.makedirs(os.path.dirname(args.out), exist_ok=True)
+    with open(args.out, "w") as f:
+        json.dump(out, f, indent=1)
+    print(json.dumps({k: v for k, v in out.items() if k != "C_iter_samples"}))
+
+
+def sweep_tiles(nd, limit):
+    """A bounded grid of feasible tiles (x threads choices): the B200 analogue of
+    the paper's baseline experiments (85 tiles x 10 thread counts)."""
+    if nd == 2:
+        tiles = [(tT, tS1, tS2, 0) for tT in (4, 8, 12, 16, 24, 32) for tS1 in (4, 8, 12, 16, 20, 28)
+                 for tS2 in (128, 256, 512)]
+    else:
+        tiles = [(tT, tS1, tS2, tS3) for tT in (2, 4, 8) for tS1 in (2, 4, 8) for tS2 in (2, 4, 8)
+                 for tS3 in (32, 64)]
+    out = []
+    for t in tiles:
+        base = t[2] // 4 if nd == 2 else (t[3] // 4) * t[2]
+        for threads in sorted({base * g for g in (1, 2, 4, 8) if base * g <= 512}):
+            try:
+                hhc.stencil_tile_resources(nd, t, threads)
+            except hhc.StencilError:
+                continue
+            out.append((t, threads))
+    random.Random(5).shuffle(out)
+    return out[:limit]
+
+
+def stats(points, key):
+    errs = [((p[key] - p["texec"]) / p["texec"]) for p in points if math.isfinite(p[key])]
+    rmse_all = math.sqrt(sum(e * e for e in errs) / len(errs)) if errs else None
+    best = min(p["texec"] for p in points)
+    near = [((p[key] - p["texec"]) / p["texec"]) for p in points
+            if p["texec"] <= 1.25 * best and math.isfinite(p[key])]
+    rmse_near = math.sqrt(sum(e * e for e in near) / len(near)) if near else None
+    return rmse_all, rmse_near, len(near)
+
+
+def sweep(args):
+    import torch
+
+    import bench
+    from synth import CONFIG_SEEDS, field
+    cfg = bench.CONFIGS[args.config]
+    kind, dims, T = cfg["kind"], cfg["dims"], cfg["T"]
+    nd = len(dims)
+    cal = load_cal(args.cal)
+    a = field(CONFIG_SEEDS[args.config], dims)
+    d_in = torch.from_numpy(a).cuda()
+    d_out = torch.empty_like(d_in)
+    h = hhc.stencil_create(kind, dims)
+    pts = []
+    t_start = time.time()
+    for tile, threads in sweep_tiles(nd, args.limit):
+        if time.time() - t_start > args.budget:
+            break
+        try:
+            te = time_run(h, d_in, d_out, T, tile, threads, reps=args.reps)
+        except hhc.StencilError:
+            continue
+        p = {"tile": list(tile), "threads": threads, "texec": te}
+        for geom, name in ((hhc.PAPER, "talg_paper"), (hhc.EXACT, "talg_exact")):
+            p[name] = hhc.model_predict(kind, dims, T, tile, b200_hw(cal, kind, geom, threads))
+        pts.append(p)
+        print(json.dumps(p), flush=True)
+    best = min(pts, key=lambda p: p["texec"])
+    res = {"config": args.config, "n_points": len(pts), "best_measured": best, "points": pts}
+    for name in ("talg_paper", "talg_exact"):
+        ra, rn, nn = stats(pts, name)
+        res[name] = {"rmse_all": ra, "rmse_within_20pct": rn, "n_within_20pct": nn}
+    # chosen-tile gaps (reading Q17), model argmin over the swept points and over Eq. 31's space
+    for geom, name in ((hhc.PAPER, "paper"), (hhc.EXACT, "exact")):
+        hw = b200_hw(cal, kind, geom)
+        try:
+            bt, bthr, cands = hhc.model_select_tile(kind, dims, T, hw, 0.10)
+            te = time_run(h, d_in, d_out, T, bt, bthr, reps=args.reps)
+            res[f"argmin_{name}"] = {"tile": list(bt), "threads": bthr, "texec": te,
+                                     "gap_vs_best_measured": te / best["texec"] - 1.0,
+                                     "n_within_10pct": len(cands)}
+        except hhc.StencilError as e:
+            res[f"argmin_{name}"] = {"error": str(e)}
+    out = args.out or os.path.join(ROOT, "profiles", f"sweep_{args.config}_r01.json")
+    with open(out, "w") as f:
+        json.dump(res, f, indent=1)
+    print(json.dumps({k: v for k, v in res.items() if k != "points"}))
+
+
+def select(args):
+    """§6.1: enumerate Eq. 31, measure every tile within `within` of Talg_min."""
+    import torch
+
+    import bench
+    from synth import CONFIG_SEEDS, field
+    cfg = bench.CONFIGS[args.config]
+    kind, dims, T = cfg["kind"], cfg["dims"], cfg["T"]
+    cal = load_cal(args.cal)
+    hw = b200_hw(cal, kind, hhc.EXACT)
+    t0 = time.time()
+    best, thr, cands = hhc.model_select_tile(kind, dims, T, hw, args.within)
+    t_sel = time.time() - t0
+    a = field(CONFIG_SEEDS[args.config], dims)
+    d_in = torch.from_numpy(a).cuda()
+    d_out = torch.empty_like(d_in)
+    h = hhc.stencil_create(kind, dims)
+    meas = []
+    cands = sorted(cands, key=lambda c: hhc.model_predict(kind, dims, T, c, hw))
+    for c in cands[:args.max_measure]:
+        try:
+            meas.append({"tile": list(c), "texec": time_run(h, d_in, d_out, T, c, 0, reps=args.reps),
+                         "talg": hhc.model_predict(kind, dims, T, c, hw)})
+        except hhc.StencilError:
+            continue
+    win = min(meas, key=lambda m: m["texec"])
+    res = {"config": args.config, "argmin": list(best), "argmin_threads": thr, "n_candidates": len(cands),
+           "enumeration_seconds": t_sel, "measured": meas, "best_within": win}
+    out = args.out or os.path.join(ROOT, "profiles", f"select_{args.config}_r01.json")
+    with open(out, "w") as f:
+        json.dump(res, f, indent=1)
+    print(json.dumps({k: v for k, v in res.items() if k != "measured"}))
+
+
+def main(argv=None):
+    ap = argparse.ArgumentParser()
+    sub = ap.add_subparsers(dest="cmd", required=True)
+    c = sub.add_parser("calibrate")
+    c.add_argument("--out", default=os.path.join(ROOT, "profiles", "hw_params_b200.json"))
+    c.add_argument("--instances", type=int, default=70)
+    s = sub.add_parser("sweep")
+    s.add_argument("--config", default="C2")
+    s.add_argument("--cal", default=None)
+    s.add_argument("--out", default=None)
+    s.add_argument("--limit", type=int, default=400)
+    s.add_argument("--reps", type=int, default=3)
+    s.add_argument("--budget", type=float, default=900.0)
+    e = sub.add_parser("select")
+    e.add_argument("--config", default="C2")
+    e.add_argument("--cal", default=None)
+    e.add_argument("--out", default=None)
+    e.add_argument("--within", type=float, default=0.10)
+    e.add_argument("--reps", type=int, default=3)
+    e.add_argument("--max-measure", type=int, default=60)
+    args = ap.parse_args(argv)
+    {"calibrate": calibrate, "sweep": sweep, "select": select}[args.cmd](args)
+
+
+if __name__ == "__main__":
+    main()

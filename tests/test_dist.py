@@ -1,0 +1,80 @@
+"""Multi-process (gloo, CPU) tests of the slab decomposition driver
+(paper_conf_ppopp_prajapatirradg17_b200/dist.py): partition, ghost
+exchange and the time-tile loop, with the CPU oracle as the per-tile stepper.
+The gathered owned rows must equal the single-domain oracle bit for bit."""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+import oracle
+from paper_conf_ppopp_prajapatirradg17_b200 import dist as hdist
+from synth import field
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _worker(rank, world, port, kind, dims, T, tT, seed, outdir):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    slab = hdist.partition(dims[0], world, rank, tT)
+    init = field(seed, dims, row_start=slab.e0, nrows=slab.rows)
+    p0 = torch.from_numpy(init.copy())
+    p1 = torch.empty_like(p0)
+
+    def step(a, b, Tt):
+        res = torch.from_numpy(oracle.run(kind, a.numpy(), Tt, oracle.FUSED))
+        if Tt % 2 == 0:
+            a.copy_(res)
+            return a
+        b.copy_(res)
+        return b
+
+    out = hdist.run_slabs(slab, p0, p1, T, tT, step, dist)
+    lo, hi = slab.held
+    np.save(os.path.join(outdir, f"r{rank}.npy"), out[lo - slab.e0:hi - slab.e0].numpy())
+    np.save(os.path.join(outdir, f"rows{rank}.npy"), np.array([lo, hi]))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world,kind,dims,T,tT", [
+    (2, oracle.HEAT2D_9PT, (41, 37), 13, 4),
+    (3, oracle.GRADIENT2D, (50, 29), 9, 2),
+    (2, oracle.JACOBI2D_5PT, (34, 40), 8, 8),
+    (2, oracle.HEAT3D_7PT, (22, 9, 11), 7, 2),
+    (3, oracle.LAPLACIAN3D_27PT, (26, 8, 7), 6, 4),
+])
+def test_slab_decomposition_matches_oracle(tmp_path, world, kind, dims, T, tT):
+    port = _free_port()
+    mp.spawn(_worker, args=(world, port, kind, dims, T, tT, 77, str(tmp_path)), nprocs=world, join=True)
+    full = oracle.run(kind, field(77, dims), T, oracle.FUSED)
+    got = np.empty_like(full)
+    covered = np.zeros(dims[0], bool)
+    for r in range(world):
+        lo, hi = np.load(tmp_path / f"rows{r}.npy")
+        got[lo:hi] = np.load(tmp_path / f"r{r}.npy")
+        assert not covered[lo:hi].any()
+        covered[lo:hi] = True
+    assert covered.all()
+    assert np.array_equal(got.view(np.uint32), full.view(np.uint32))
+
+
+def test_partition_rules():
+    s = hdist.partition(8194, 8, 0, 16)
+    assert (s.r0, s.e0, s.held) == (1, 0, (0, s.r1))
+    s7 = hdist.partition(8194, 8, 7, 16)
+    assert s7.r1 == 8193 and s7.e1 == 8194 and s7.held[1] == 8194
+    with pytest.raises(ValueError):
+        hdist.partition(40, 8, 0, 16)            # slabs thinner than the ghost depth

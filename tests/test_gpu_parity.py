@@ -217,3 +217,46 @@ def test_full_size_closed_forms(cfg, kind, dims, T):
     for x0 in range(0, dims[0], 64):                  # slab-wise, bounded host memory
         ex = (lam ** T) * sines[0][x0:x0 + 64].reshape([-1] + [1] * (nd - 1)) * rest[None]
         assert np.max(np.abs(got[x0:x0 + 64].astype(np.float64) - ex)) <= tol, (cfg, lam, x0)
+
+
+@pytest.mark.parametrize("kind,dims,T,tT,nslab", [
+    (hhc.HEAT2D_9PT, (131, 150), 37, 8, 3),
+    (hhc.GRADIENT2D, (90, 77), 21, 4, 2),
+    (hhc.HEAT3D_7PT, (40, 30, 70), 11, 4, 2),
+    (hhc.LAPLACIAN3D_27PT, (45, 22, 40), 9, 2, 3),
+])
+def test_virtual_slabs_run_planes(kind, dims, T, tT, nslab):
+    """The multi-GPU time-tile loop (dist.partition + stencil_run_planes) with
+    `nslab` virtual ranks on one GPU; ghosts are exchanged by device copies in
+    the same pattern as dist.exchange.  Owned rows must equal the oracle."""
+    from paper_conf_ppopp_prajapatirradg17_b200 import dist as hdist
+    a = field(99, dims)
+    tile = (tT, 3, 32) if len(dims) == 2 else (tT, 2, 3, 32)
+    slabs = [hdist.partition(dims[0], nslab, r, tT) for r in range(nslab)]
+    hs = [hhc.stencil_create(kind, (s.rows,) + dims[1:]) for s in slabs]
+    p0 = [torch.from_numpy(np.ascontiguousarray(a[s.e0:s.e1])).to(DEV) for s in slabs]
+    p1 = [torch.empty_like(x) for x in p0]
+    cur = list(p0)
+    done = 0
+    while done < T:
+        Tt = min(tT, T - done)
+        for r, s in enumerate(slabs):            # ghost exchange (the dist.exchange pattern)
+            lo, hi = s.r0 - s.e0, s.r1 - s.e0
+            if r > 0:
+                sp = slabs[r - 1]
+                cur[r][lo - tT:lo] = cur[r - 1][sp.r1 - sp.e0 - tT:sp.r1 - sp.e0]
+            if r < nslab - 1:
+                sn = slabs[r + 1]
+                cur[r][hi:hi + tT] = cur[r + 1][sn.r0 - sn.e0:sn.r0 - sn.e0 + tT]
+        torch.cuda.synchronize()
+        for r in range(nslab):
+            other = p1[r] if cur[r] is p0[r] else p0[r]
+            hhc.stencil_run_planes(hs[r], slabs[r].rows, cur[r], other, Tt, tile)
+            cur[r] = cur[r] if Tt % 2 == 0 else other
+        torch.cuda.synchronize()
+        done += Tt
+    exp = oracle.run(kind, a, T, hhc.FUSED)
+    for r, s in enumerate(slabs):
+        lo, hi = s.held
+        got = cur[r][lo - s.e0:hi - s.e0].cpu().numpy()
+        assert_bits(np.ascontiguousarray(got), np.ascontiguousarray(exp[lo:hi]), f"slab {r}")
