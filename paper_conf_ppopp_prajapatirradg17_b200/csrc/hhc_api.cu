@@ -205,16 +205,6 @@ static int check_tile(int ndims, stencil_tile t, int threads, int smem_limit, in
     return STENCIL_OK;
 }
 
-// K1R eligibility: 2D, default weights, hexagon rows fit
-// the register rows, whole warps of 4-column threads, threads = tS2/4.
-static int reg_choice(stencil_t h, const stencil_tile& t, int threads) {
-    if (h->ndims != 2 || !h->defw || getenv("HHC_NO_REG")) return 0;
-    const int nr = reg_rows_for(t.s1 + t.t + 2);
-    if (!nr || t.s2 % 128 || t.s2 > 1024) return 0;
-    if (threads != 0 && threads != t.s2 / 4) return 0;
-    return nr;
-}
-
 extern "C" int stencil_tile_resources(int ndims, stencil_tile tile, int threads, int64_t* smem,
                                       int* block_threads, int* regs) {
     if (ndims != 2 && ndims != 3) return STENCIL_EINVAL;
@@ -290,11 +280,10 @@ static int choose_J(stencil_t h, const RowPlan& r) {
 // Everything that must not happen inside stream capture: the kernel's smem
 // attribute, its occupancy (for J), and the 3D flag buffer.
 static int prepare_rows(stencil_t h, const int64_t* dims, int64_t T, stencil_tile tile, int thr, int nr = 0) {
-    hex_kernel_t k = nr ? get_hex_reg_kernel(h->kind, h->mode, nr)
-                        : get_hex_kernel(h->ndims, h->kind, h->mode, h->has_c, h->defw);
+    (void)nr;
+    hex_kernel_t k = get_hex_kernel(h->ndims, h->kind, h->mode, h->has_c, h->defw);
     if (!k) return STENCIL_EINVAL;
-    const int64_t smem = nr ? smem_bytes_reg(tile.t, tile.s2, nr)
-                            : smem_bytes(h->ndims, tile.t, tile.s1, tile.s2, tile.s3);
+    const int64_t smem = smem_bytes(h->ndims, tile.t, tile.s1, tile.s2, tile.s3);
     cudaError_t e = cudaFuncSetAttribute((const void*)k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return cuda_fail(h, e);
     if (h->ndims != 3) return STENCIL_OK;
@@ -328,12 +317,10 @@ static int enqueue_rows(stencil_t h, const int64_t* dims, const float* ring, flo
                         std::vector<cudaEvent_t>* evs = nullptr, int nr = 0) {
     std::vector<RowPlan> rows;
     plan_rows(h->ndims, dims, T, tile, rows);
-    hex_kernel_t k = nr ? get_hex_reg_kernel(h->kind, h->mode, nr)
-                        : get_hex_kernel(h->ndims, h->kind, h->mode, h->has_c, h->defw);
+    (void)nr;
+    hex_kernel_t k = get_hex_kernel(h->ndims, h->kind, h->mode, h->has_c, h->defw);
     if (!k) return STENCIL_EINVAL;
-    const int64_t smem = nr ? smem_bytes_reg(tile.t, tile.s2, nr)
-                            : smem_bytes(h->ndims, tile.t, tile.s1, tile.s2, tile.s3);
-    if (nr) { thr = tile.s2 / 4; G = 1; }
+    const int64_t smem = smem_bytes(h->ndims, tile.t, tile.s1, tile.s2, tile.s3);
     int64_t nl = 0;
     cudaError_t e;
     // 3D: thread blocks per slab J (pipelined along S2, flags in global memory);
@@ -481,7 +468,7 @@ extern "C" int stencil_run(stencil_t h, const float* d_in, float* d_out, int64_t
         if (e != cudaSuccess) { h->scratch = nullptr; return STENCIL_ENOMEM; }
     }
     r.planes_mode = 0; r.a = d_in; r.b = d_out;
-    r.nr = reg_choice(h, tile, threads);
+    r.nr = 0;
     for (int d = 0; d < 3; ++d) r.dims[d] = h->dims[d];
     r.T = T; r.tile = tile;
     if (h->ndims == 2) r.tile.s3 = 0;
@@ -498,7 +485,7 @@ extern "C" int stencil_run_planes(stencil_t h, int64_t rows, float* plane0, floa
     if (rc) return rc;
     cudaSetDevice(h->device);
     r.planes_mode = 1; r.a = plane0; r.b = plane1;
-    r.nr = reg_choice(h, tile, threads);
+    r.nr = 0;
     r.dims[0] = rows; r.dims[1] = h->dims[1]; r.dims[2] = h->dims[2];
     const int64_t n = r.dims[0] * r.dims[1] * r.dims[2];
     if (plane1 < plane0 + n && plane0 < plane1 + n) return STENCIL_EINVAL;
@@ -548,7 +535,7 @@ extern "C" int stencil_profile(stencil_t h, const float* d_in, float* d_out, int
     plane[1 - (T & 1)] = h->scratch;
     launch_copy_full(d_in, plane[0], n, s);
     launch_copy_ring(d_in, plane[1], h->dims[0], h->dims[1], h->dims[2], s);
-    const int nr = reg_choice(h, tile, threads);
+    const int nr = 0;
     rc = prepare_rows(h, h->dims, T, tile, thr, nr);
     if (rc) return rc;
     std::vector<cudaEvent_t> evs;

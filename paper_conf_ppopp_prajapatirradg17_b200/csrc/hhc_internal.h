@@ -47,15 +47,7 @@ inline int column_threads(int ndims, int tS2, int tS3) {
     return ndims == 2 ? tS2 / kCols2D : (tS3 / kCols3D) * tS2;
 }
 
-// K1R (register-resident 2D kernel): register rows NR >= tS1+tT+2, threads = tS2/4.
-inline int64_t smem_bytes_reg(int tT, int tS2, int NR) {
-    const int64_t nw = tS2 / 128;
-    return 4 * (2 * 4 * (int64_t)tS2 + 2 * nw * NR * 2 + 2 * (int64_t)(tT + 1) * NR * 2 + 16 * (int64_t)tT);
-}
-
 typedef void (*hex_kernel_t)(HexParams);
-hex_kernel_t get_hex_reg_kernel(int kind, int mode, int nr);
-int reg_rows_for(int NX);
 hex_kernel_t get_hex_kernel(int ndims, int kind, int mode, bool has_c, bool defw);
 int hex_kernel_regs(int ndims, int kind, int mode, bool has_c, bool defw);
 void launch_copy_ring(const float* in, float* out, int64_t S1, int64_t S2, int64_t S3, void* stream);

@@ -261,21 +261,3 @@ def test_virtual_slabs_run_planes(kind, dims, T, tT, nslab):
         got = cur[r][lo - s.e0:hi - s.e0].cpu().numpy()
         assert_bits(np.ascontiguousarray(got), np.ascontiguousarray(exp[lo:hi]), f"slab {r}")
 
-
-REG_TILES = [(2, 1, 128), (4, 3, 128), (8, 5, 256), (16, 4, 128), (6, 2, 512), (10, 7, 128), (16, 20, 512),
-             (12, 26, 128), (22, 14, 256), (2, 13, 1024)]
-
-
-@pytest.mark.parametrize("kind", [hhc.JACOBI2D_5PT, hhc.HEAT2D_9PT, hhc.GRADIENT2D, hhc.LAPLACIAN2D_5PT])
-@pytest.mark.parametrize("mode", [hhc.PLAIN, hhc.FUSED])
-def test_parity_register_kernel(kind, mode):
-    """K1R (register-resident 2D kernel; default weights, tS2 % 128 == 0,
-    tS1+tT+2 <= 40): random sizes incl. grids smaller than a tile, odd T."""
-    rng = np.random.default_rng(1000 + kind * 10 + mode)
-    for tile in REG_TILES:
-        dims = (int(rng.integers(3, 140)), int(rng.integers(3, 700)))
-        a = field(int(rng.integers(1, 1 << 30)), dims)
-        for T in (1, 3, tile[0] + 1, 2 * tile[0] + 3):
-            exp = oracle.run(kind, a, T, mode)
-            got = gpu_run(kind, a, T, tile, mode)
-            assert_bits(got, exp, f"K1R kind {kind} mode {mode} dims {dims} T {T} tile {tile}")
