@@ -80,7 +80,6 @@ __global__ void __launch_bounds__(512) hex2d_pair_kernel(const __grid_constant__
     const int colbase = kCW * wg + 4 * lane;           // u0 - (a - 4)
     const int s = colbase + 4;                         // smem slot of column k = 0
     const bool store_lane = lane != 0;                 // lane 0 is the overlap lane
-    const bool face_lane = (wg == nw - 1) && lane >= 30;
 
     for (int j2 = 0; j2 < p.n2; ++j2) {
         const int64_t a = 1 + (int64_t)j2 * tS2;
@@ -108,7 +107,10 @@ __global__ void __launch_bounds__(512) hex2d_pair_kernel(const __grid_constant__
                         const int64_t x = xs + pp;
                         if (l > 0 && (x == 0 || x == S1 - 1)) continue;   // ring rows: per-pass fill
                         const float* row = src + x * S2;
-                        for (int c = gtid; c < (full ? W : 6); c += 32 * nw) {
+                        // halo columns (c < 6) only in the first sub-tile: later ones take
+                        // them from the face, because global memory may already hold level
+                        // l+1 there (written by the previous sub-tile of this block)
+                        for (int c = gtid + (j2 > 0 ? 6 : 0); c < (full ? W : 6); c += 32 * nw) {
                             const int64_t y = ybase + c;
                             if (y < 0 || y >= S2) continue;
                             float* d = (c >= 6 || l == 0) ? dpl + pp * RS + c + 2 : fcur + (l * NX + pp) * 6 + c;
@@ -136,6 +138,13 @@ __global__ void __launch_bounds__(512) hex2d_pair_kernel(const __grid_constant__
             }
             cp_async_wait_all();
         }
+        if (j2 > 0) {                                   // halo of the first pass from the face
+            float* const R0 = (((sched[0] >> 4) + 1) & 1) ? pl1 : pl0;
+            for (int i = tid; i < NX * 6; i += nthr) {
+                const int pp = i / 6, c = i - pp * 6;
+                R0[pp * RS + 2 + c] = fcur[pp * 6 + c];  // level 0 entry, ring rows included
+            }
+        }
         __syncthreads();
 
         int npair = 0;                                  // pairs done in this sub-tile (stage parity)
@@ -146,9 +155,11 @@ __global__ void __launch_bounds__(512) hex2d_pair_kernel(const __grid_constant__
             const int lout = type == 2 ? l + 1 : l;     // level stored by this pass
             const int* g = geo + l * kGeo;
             // halo slots of the next pass's read plane (= Wp), from the face of level lout+1
+            // and the face of level l (its last 6 columns of level l-1) for the next sub-tile
             for (int i = tid; i < NX * 6; i += nthr) {
                 const int pp = i / 6, c = i - pp * 6;
                 const int64_t xr = xs + pp;
+                fnxt[(l * NX + pp) * 6 + c] = R[pp * RS + tS2 + 2 + c];
                 if (lout + 1 < nlev && xr != 0 && xr != S1 - 1)
                     Wp[pp * RS + 2 + c] = fcur[((lout + 1) * NX + pp) * 6 + c];
             }
@@ -197,7 +208,6 @@ __global__ void __launch_bounds__(512) hex2d_pair_kernel(const __grid_constant__
                         float* gp = p.plane[(tb + l) & 1] + (xs + pa) * S2 + y0;
                         const float* __restrict__ rp = R + (pa - 1) * RS + s;
                         float* __restrict__ wp = Wp + pa * RS + s;
-                        float* fw = fnxt + ((l + 1) * NX + pa) * 6;
                         int pp = pa;
                         auto step = [&](const float(&r0)[6], const float(&r1)[6], float(&r2)[6]) {
                             ld6(rp, r2);
@@ -215,15 +225,7 @@ __global__ void __launch_bounds__(512) hex2d_pair_kernel(const __grid_constant__
                                 }
                             }
                             if (store_lane) *reinterpret_cast<float4*>(wp) = make_float4(o[0], o[1], o[2], o[3]);
-                            if (face_lane) {
-                                if (lane == 31) {
-                                    fw[2] = o[0]; fw[3] = o[1]; fw[4] = o[2]; fw[5] = o[3];
-                                } else {
-                                    fw[0] = o[2]; fw[1] = o[3];
-                                }
-                            }
                             wp += RS;
-                            fw += 6;
                             if (store_lane && (unsigned)(pp - (int)nwlo) >= nwlen && !p.compute_only) {
 #pragma unroll
                                 for (int kk = 0; kk < 4; ++kk)
@@ -269,24 +271,18 @@ __global__ void __launch_bounds__(512) hex2d_pair_kernel(const __grid_constant__
                         float* const gpl0 = p.plane[(tb + l) & 1];
                         float* const gpl1 = p.plane[(tb + l + 1) & 1];
                         const float* __restrict__ rp = R + (a1 - 2) * RS + s;       // level l-1 row x-1 at x = a1-1
-                        // level l-1 window: rows x-1 (Pm), x (Pc); level l window: rows x-2 (Lm), x-1 (Lc)
-                        float Pm[6], Pc[6], Pn[6];
-                        float Lm[6], Lc[6], Ln[6];
-                        ld6(rp, Pm);
-                        rp += RS;
-                        ld6(rp, Pc);
-                        rp += RS;
-#pragma unroll
-                        for (int kk = 0; kk < 6; ++kk) { Lm[kk] = 0.0f; Lc[kk] = 0.0f; }
-                        for (int x = a1 - 1; x <= e1; ++x) {
-                            // -- level l, row x
-                            ld6(rp, Pn);
+                        int x = a1 - 1;
+                        // one step: level l at row x (from level l-1 rows x-1..x+1 = P0, P1, P2),
+                        // then level l+1 at row x-1 (from level l rows x-2..x = L0, L1, L2)
+                        auto pstep = [&](const float(&P0)[6], const float(&P1)[6], float(&P2)[6],
+                                         const float(&L0)[6], const float(&L1)[6], float(&L2)[6]) {
+                            ld6(rp, P2);
                             rp += RS;
                             float o[4];
                             const int64_t xg = xs + x;
                             if (x >= rl && x < rr) {
 #pragma unroll
-                                for (int kk = 0; kk < 4; ++kk) o[kk] = point2<KIND, MODE, HASC, DEFW, 6>(Pm, Pc, Pn, kk, p);
+                                for (int kk = 0; kk < 4; ++kk) o[kk] = point2<KIND, MODE, HASC, DEFW, 6>(P0, P1, P2, kk, p);
                                 if (!allv0) {
                                     const float* inrow = p.in + xg * S2;
 #pragma unroll
@@ -296,18 +292,12 @@ __global__ void __launch_bounds__(512) hex2d_pair_kernel(const __grid_constant__
                                         else if (y < 1 || y > S2i - 2) o[kk] = 0.0f;
                                     }
                                 }
-                                if (x >= own_lo && x < own_hi) {
-                                    if (face_lane) {
-                                        float* fw = fnxt + ((l + 1) * NX + x) * 6;
-                                        if (lane == 31) { fw[2] = o[0]; fw[3] = o[1]; fw[4] = o[2]; fw[5] = o[3]; }
-                                        else { fw[0] = o[2]; fw[1] = o[3]; }
-                                    }
-                                    if (store_lane && (unsigned)(x - (int)nwlo0) >= nwlen0 && !p.compute_only) {
-                                        float* gp = gpl0 + xg * S2 + y0;
+                                if (store_lane && x >= own_lo && x < own_hi &&
+                                    (unsigned)(x - (int)nwlo0) >= nwlen0 && !p.compute_only) {
+                                    float* gp = gpl0 + xg * S2 + y0;
 #pragma unroll
-                                        for (int kk = 0; kk < 4; ++kk)
-                                            if (allv0 || (y0 + kk >= 1 && y0 + kk <= S2i - 2)) gp[kk] = o[kk];
-                                    }
+                                    for (int kk = 0; kk < 4; ++kk)
+                                        if (allv0 || (y0 + kk >= 1 && y0 + kk <= S2i - 2)) gp[kk] = o[kk];
                                 }
                             } else if (xg == 0 || xg == S1 - 1) {           // ring row at the skew of level l
                                 const float* inrow = p.in + xg * S2;
@@ -318,19 +308,18 @@ __global__ void __launch_bounds__(512) hex2d_pair_kernel(const __grid_constant__
                                 }
                             } else {                                         // footprint row of level l+1
                                 const int slot = (x >= f1a && x - f1a < f1n) ? x - f1a : f1n + (x - f2a);
-                                const float4 q = *reinterpret_cast<const float4*>(st + slot * SR);
-                                o[0] = q.x; o[1] = q.y; o[2] = q.z; o[3] = q.w;
+                                const float4 q4 = *reinterpret_cast<const float4*>(st + slot * SR);
+                                o[0] = q4.x; o[1] = q4.y; o[2] = q4.z; o[3] = q4.w;
                             }
-                            Ln[0] = __shfl_up_sync(kFullMask, o[2], 1);
-                            Ln[1] = __shfl_up_sync(kFullMask, o[3], 1);
-                            Ln[2] = o[0]; Ln[3] = o[1]; Ln[4] = o[2]; Ln[5] = o[3];
-                            // -- level l+1, row x-1
+                            L2[0] = __shfl_up_sync(kFullMask, o[2], 1);
+                            L2[1] = __shfl_up_sync(kFullMask, o[3], 1);
+                            L2[2] = o[0]; L2[3] = o[1]; L2[4] = o[2]; L2[5] = o[3];
                             const int xm = x - 1;
                             if (xm >= a1) {
                                 float q[4];
 #pragma unroll
-                                for (int kk = 0; kk < 4; ++kk) q[kk] = point2<KIND, MODE, HASC, DEFW, 6>(Lm, Lc, Ln, kk, p);
-                                const int64_t xmg = xs + xm;
+                                for (int kk = 0; kk < 4; ++kk) q[kk] = point2<KIND, MODE, HASC, DEFW, 6>(L0, L1, L2, kk, p);
+                                const int64_t xmg = xg - 1;
                                 if (!allv1) {
                                     const float* inrow = p.in + xmg * S2;
 #pragma unroll
@@ -342,11 +331,6 @@ __global__ void __launch_bounds__(512) hex2d_pair_kernel(const __grid_constant__
                                 }
                                 if (store_lane)
                                     *reinterpret_cast<float4*>(Wp + xm * RS + s) = make_float4(q[0], q[1], q[2], q[3]);
-                                if (face_lane) {
-                                    float* fw = fnxt + ((l + 2) * NX + xm) * 6;
-                                    if (lane == 31) { fw[2] = q[0]; fw[3] = q[1]; fw[4] = q[2]; fw[5] = q[3]; }
-                                    else { fw[0] = q[2]; fw[1] = q[3]; }
-                                }
                                 if (store_lane && (unsigned)(xm - (int)nwlo1) >= nwlen1 && !p.compute_only) {
                                     float* gp = gpl1 + xmg * S2 + y1;
 #pragma unroll
@@ -354,12 +338,23 @@ __global__ void __launch_bounds__(512) hex2d_pair_kernel(const __grid_constant__
                                         if (allv1 || (y1 + kk >= 1 && y1 + kk <= S2i - 2)) gp[kk] = q[kk];
                                 }
                             }
+                            ++x;
+                        };
+                        float PA[6], PB[6], PC[6], LA[6], LB[6], LC[6];
+                        ld6(rp, PA);
+                        rp += RS;
+                        ld6(rp, PB);
+                        rp += RS;
 #pragma unroll
-                            for (int kk = 0; kk < 6; ++kk) {
-                                Pm[kk] = Pc[kk]; Pc[kk] = Pn[kk];
-                                Lm[kk] = Lc[kk]; Lc[kk] = Ln[kk];
-                            }
+                        for (int kk = 0; kk < 6; ++kk) { LA[kk] = 0.0f; LB[kk] = 0.0f; }
+                        int n = e1 - a1 + 2;                                 // steps x = a1-1 .. e1
+                        for (; n >= 3; n -= 3) {                             // rotating names, no moves
+                            pstep(PA, PB, PC, LA, LB, LC);
+                            pstep(PB, PC, PA, LB, LC, LA);
+                            pstep(PC, PA, PB, LC, LA, LB);
                         }
+                        if (n >= 1) pstep(PA, PB, PC, LA, LB, LC);
+                        if (n >= 2) pstep(PB, PC, PA, LB, LC, LA);
                     }
                 }
             }
