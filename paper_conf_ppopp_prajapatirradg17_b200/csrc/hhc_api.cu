@@ -184,7 +184,7 @@ extern "C" void stencil_destroy(stencil_t h) {
 static int check_tile(int ndims, stencil_tile t, int threads, int smem_limit, int* G_out, int* thr_out) {
     if (t.t < 2 || (t.t & 1) || t.s1 < 1) return STENCIL_ETILE;
     if (ndims == 2) {
-        if (t.s2 < 32 || (t.s2 % 32 && !is_pair_tile(ndims, t.s2))) return STENCIL_ETILE;
+        if (t.s2 < 32 || t.s2 % 32) return STENCIL_ETILE;
     } else {
         if (t.s2 < 1 || t.s3 < 32 || t.s3 % 32) return STENCIL_ETILE;
     }
@@ -198,8 +198,7 @@ static int check_tile(int ndims, stencil_tile t, int threads, int smem_limit, in
         if (threads < 0 || threads > 512 || threads % base) return STENCIL_EINVAL;
         G = threads / base;
     }
-    const int64_t sm = is_pair_tile(ndims, t.s2) ? smem_bytes_pair(t.t, t.s1, t.s2)
-                                                 : smem_bytes(ndims, t.t, t.s1, t.s2, t.s3);
+    const int64_t sm = smem_bytes(ndims, t.t, t.s1, t.s2, t.s3);
     if (sm > smem_limit) return STENCIL_ETILE;
     *G_out = G;
     *thr_out = base * G;
@@ -212,8 +211,7 @@ extern "C" int stencil_tile_resources(int ndims, stencil_tile tile, int threads,
     int G, thr;
     const int rc = check_tile(ndims, tile, threads, 227 * 1024, &G, &thr);
     if (rc) return rc;
-    if (smem) *smem = is_pair_tile(ndims, tile.s2) ? smem_bytes_pair(tile.t, tile.s1, tile.s2)
-                                                   : smem_bytes(ndims, tile.t, tile.s1, tile.s2, tile.s3);
+    if (smem) *smem = smem_bytes(ndims, tile.t, tile.s1, tile.s2, tile.s3);
     if (block_threads) *block_threads = thr;
     if (regs) *regs = 0;
     return STENCIL_OK;
@@ -283,12 +281,9 @@ static int choose_J(stencil_t h, const RowPlan& r) {
 // attribute, its occupancy (for J), and the 3D flag buffer.
 static int prepare_rows(stencil_t h, const int64_t* dims, int64_t T, stencil_tile tile, int thr, int nr = 0) {
     (void)nr;
-    const bool pair = is_pair_tile(h->ndims, tile.s2);
-    hex_kernel_t k = pair ? get_hex_pair_kernel(h->kind, h->mode, h->has_c, h->defw)
-                          : get_hex_kernel(h->ndims, h->kind, h->mode, h->has_c, h->defw);
+    hex_kernel_t k = get_hex_kernel(h->ndims, h->kind, h->mode, h->has_c, h->defw);
     if (!k) return STENCIL_EINVAL;
-    const int64_t smem = pair ? smem_bytes_pair(tile.t, tile.s1, tile.s2)
-                              : smem_bytes(h->ndims, tile.t, tile.s1, tile.s2, tile.s3);
+    const int64_t smem = smem_bytes(h->ndims, tile.t, tile.s1, tile.s2, tile.s3);
     cudaError_t e = cudaFuncSetAttribute((const void*)k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return cuda_fail(h, e);
     if (h->ndims != 3) return STENCIL_OK;
@@ -323,12 +318,9 @@ static int enqueue_rows(stencil_t h, const int64_t* dims, const float* ring, flo
     std::vector<RowPlan> rows;
     plan_rows(h->ndims, dims, T, tile, rows);
     (void)nr;
-    const bool pair = is_pair_tile(h->ndims, tile.s2);
-    hex_kernel_t k = pair ? get_hex_pair_kernel(h->kind, h->mode, h->has_c, h->defw)
-                          : get_hex_kernel(h->ndims, h->kind, h->mode, h->has_c, h->defw);
+    hex_kernel_t k = get_hex_kernel(h->ndims, h->kind, h->mode, h->has_c, h->defw);
     if (!k) return STENCIL_EINVAL;
-    const int64_t smem = pair ? smem_bytes_pair(tile.t, tile.s1, tile.s2)
-                              : smem_bytes(h->ndims, tile.t, tile.s1, tile.s2, tile.s3);
+    const int64_t smem = smem_bytes(h->ndims, tile.t, tile.s1, tile.s2, tile.s3);
     int64_t nl = 0;
     cudaError_t e;
     // 3D: thread blocks per slab J (pipelined along S2, flags in global memory);

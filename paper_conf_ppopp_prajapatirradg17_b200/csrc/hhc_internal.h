@@ -43,21 +43,11 @@ inline int64_t smem_bytes(int ndims, int tT, int tS1, int tS2, int tS3) {
     return 4 * (2 * NX * (tS2 + 2) * (tS3 + 4) + 2 * (int64_t)tT * NX * (tS2 + 2) * 2 + geo);
 }
 
-// K1P (two levels per shared-memory pass, 2D): tS2 = 124 * warps per x-group.
-constexpr int kPairCW = 124;
-inline bool is_pair_tile(int ndims, int tS2) { return ndims == 2 && tS2 >= kPairCW && tS2 % kPairCW == 0; }
-inline int64_t smem_bytes_pair(int tT, int tS1, int tS2) {
-    const int64_t NX = tS1 + tT + 2, RS = tS2 + 8;
-    return 4 * (2 * (NX + 2) * RS + 2 * (int64_t)(tT + 1) * NX * 6 + 2 * 4 * (int64_t)(tS2 + 4) + 17 * (int64_t)tT);
-}
-
 inline int column_threads(int ndims, int tS2, int tS3) {
-    if (is_pair_tile(ndims, tS2)) return 32 * (tS2 / kPairCW);
     return ndims == 2 ? tS2 / kCols2D : (tS3 / kCols3D) * tS2;
 }
 
 typedef void (*hex_kernel_t)(HexParams);
-hex_kernel_t get_hex_pair_kernel(int kind, int mode, bool has_c, bool defw);
 hex_kernel_t get_hex_kernel(int ndims, int kind, int mode, bool has_c, bool defw);
 int hex_kernel_regs(int ndims, int kind, int mode, bool has_c, bool defw);
 void launch_copy_ring(const float* in, float* out, int64_t S1, int64_t S2, int64_t S3, void* stream);

@@ -262,31 +262,3 @@ def test_virtual_slabs_run_planes(kind, dims, T, tT, nslab):
         assert_bits(np.ascontiguousarray(got), np.ascontiguousarray(exp[lo:hi]), f"slab {r}")
 
 
-
-PAIR_TILES = [((2, 1, 124), 0), ((4, 3, 124), 64), ((8, 5, 248), 0), ((16, 4, 124), 128), ((6, 2, 496), 256),
-              ((10, 7, 124), 32), ((16, 20, 496), 512), ((12, 26, 248), 64), ((22, 14, 372), 384), ((2, 13, 992), 256),
-              ((3 * 2, 9, 620), 160)]
-
-
-@pytest.mark.parametrize("kind", [hhc.JACOBI2D_5PT, hhc.HEAT2D_9PT, hhc.GRADIENT2D, hhc.LAPLACIAN2D_5PT])
-@pytest.mark.parametrize("mode", [hhc.PLAIN, hhc.FUSED])
-def test_parity_pair_kernel(kind, mode):
-    """K1P (two levels per shared-memory pass; tS2 = 124 * warps): random sizes
-    incl. grids smaller than a tile, odd T (single-level tail), x-groups."""
-    rng = np.random.default_rng(2000 + kind * 10 + mode)
-    for tile, threads in PAIR_TILES:
-        dims = (int(rng.integers(3, 140)), int(rng.integers(3, 1300)))
-        a = field(int(rng.integers(1, 1 << 30)), dims)
-        for T in (1, 2, 3, tile[0] + 1, 2 * tile[0] + 3):
-            exp = oracle.run(kind, a, T, mode)
-            got = gpu_run(kind, a, T, tile, mode, threads=threads)
-            assert_bits(got, exp, f"K1P kind {kind} mode {mode} dims {dims} T {T} tile {tile} thr {threads}")
-
-
-def test_pair_kernel_custom_coeffs():
-    a = field(8, (90, 400))
-    offs, w = oracle.stencil_info(hhc.HEAT2D_9PT)
-    coeffs = [float(x) * 0.9 for x in w] + [0.01]
-    for mode in (hhc.PLAIN, hhc.FUSED):
-        exp = oracle.run(hhc.HEAT2D_9PT, a, 13, mode, coeffs=coeffs)
-        assert_bits(gpu_run(hhc.HEAT2D_9PT, a, 13, (4, 3, 248), mode, coeffs=coeffs), exp, f"coeffs {mode}")
