@@ -43,13 +43,16 @@ inline int64_t smem_bytes(int ndims, int tT, int tS1, int tS2, int tS3) {
     return 4 * (2 * NX * (tS2 + 2) * (tS3 + 4) + 2 * (int64_t)tT * NX * (tS2 + 2) * 2 + geo);
 }
 
+// 2D column groups per thread (K1): two groups 128 columns apart when tS2 % 256 == 0.
+inline int col_groups_2d(int tS2) { return tS2 % 256 == 0 ? 2 : 1; }
+
 inline int column_threads(int ndims, int tS2, int tS3) {
-    return ndims == 2 ? tS2 / kCols2D : (tS3 / kCols3D) * tS2;
+    return ndims == 2 ? tS2 / (kCols2D * col_groups_2d(tS2)) : (tS3 / kCols3D) * tS2;
 }
 
 typedef void (*hex_kernel_t)(HexParams);
-hex_kernel_t get_hex_kernel(int ndims, int kind, int mode, bool has_c, bool defw);
-int hex_kernel_regs(int ndims, int kind, int mode, bool has_c, bool defw);
+hex_kernel_t get_hex_kernel(int ndims, int kind, int mode, bool has_c, bool defw, int ng);
+int hex_kernel_regs(int ndims, int kind, int mode, bool has_c, bool defw, int ng);
 void launch_copy_ring(const float* in, float* out, int64_t S1, int64_t S2, int64_t S3, void* stream);
 void launch_copy_full(const float* in, float* out, int64_t n, void* stream);
 
