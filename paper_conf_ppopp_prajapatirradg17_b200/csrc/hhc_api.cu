@@ -281,7 +281,7 @@ static int choose_J(stencil_t h, const RowPlan& r) {
 // attribute, its occupancy (for J), and the 3D flag buffer.
 static int prepare_rows(stencil_t h, const int64_t* dims, int64_t T, stencil_tile tile, int thr, int nr = 0) {
     (void)nr;
-    hex_kernel_t k = get_hex_kernel(h->ndims, h->kind, h->mode, h->has_c, h->defw, h->ndims == 2 ? col_groups_2d(tile.s2) : 1);
+    hex_kernel_t k = get_hex_kernel(h->ndims, h->kind, h->mode, h->has_c, h->defw);
     if (!k) return STENCIL_EINVAL;
     const int64_t smem = smem_bytes(h->ndims, tile.t, tile.s1, tile.s2, tile.s3);
     cudaError_t e = cudaFuncSetAttribute((const void*)k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
@@ -318,7 +318,7 @@ static int enqueue_rows(stencil_t h, const int64_t* dims, const float* ring, flo
     std::vector<RowPlan> rows;
     plan_rows(h->ndims, dims, T, tile, rows);
     (void)nr;
-    hex_kernel_t k = get_hex_kernel(h->ndims, h->kind, h->mode, h->has_c, h->defw, h->ndims == 2 ? col_groups_2d(tile.s2) : 1);
+    hex_kernel_t k = get_hex_kernel(h->ndims, h->kind, h->mode, h->has_c, h->defw);
     if (!k) return STENCIL_EINVAL;
     const int64_t smem = smem_bytes(h->ndims, tile.t, tile.s1, tile.s2, tile.s3);
     int64_t nl = 0;

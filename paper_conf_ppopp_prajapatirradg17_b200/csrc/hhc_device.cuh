@@ -104,6 +104,31 @@ __device__ __forceinline__ float grad2(const float (&r0)[N], const float (&r1)[N
     return __fadd_rn(c, q);
 }
 
+// Packed pair form of lin2 (K1 pair layout): every row register holds the two
+// columns (q, q + D) of one pair, so each stencil term of both points is one
+// f32x2 operation on an aligned register pair (FFMA2/FMUL2 on sm_100a).  Each
+// half is the same correctly rounded operation sequence as lin2 (reading R4),
+// hence bit-identical.  Only for MODE_FUSED: ptxas contracts a packed
+// mul.rn + add.rn pair into FFMA2 (observed with CUDA 12.9), so the plain mode
+// keeps scalar __fmul_rn/__fadd_rn.
+template <int KIND, bool DEFW, int J>
+__device__ __forceinline__ float2 lin_term2x2(float2 acc, const float2 (&r0)[6], const float2 (&r1)[6],
+                                              const float2 (&r2)[6], int k, const HexParams& p) {
+    constexpr Off o = kind_off(KIND, J);
+    const float2 v = o.d1 < 0 ? r0[k + 1 + o.d2] : o.d1 == 0 ? r1[k + 1 + o.d2] : r2[k + 1 + o.d2];
+    const float w = wgt<KIND, DEFW, J>(p);
+    if constexpr (J == 0) return __fmul2_rn(make_float2(w, w), v);
+    else return __ffma2_rn(make_float2(w, w), v, acc);
+}
+template <int KIND, bool HASC, bool DEFW, int... J>
+__device__ __forceinline__ float2 lin2x2(const float2 (&r0)[6], const float2 (&r1)[6], const float2 (&r2)[6], int k,
+                                         const HexParams& p, std::integer_sequence<int, J...>) {
+    float2 acc = make_float2(0.0f, 0.0f);
+    ((acc = lin_term2x2<KIND, DEFW, J>(acc, r0, r1, r2, k, p)), ...);
+    if constexpr (HASC) acc = __fadd2_rn(acc, make_float2(p.c, p.c));
+    return acc;
+}
+
 template <int KIND, int MODE, bool HASC, bool DEFW, int N>
 __device__ __forceinline__ float point2(const float (&r0)[N], const float (&r1)[N], const float (&r2)[N], int k,
                                         const HexParams& p) {

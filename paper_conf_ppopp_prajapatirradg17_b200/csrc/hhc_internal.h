@@ -7,7 +7,6 @@
 
 namespace hhc {
 
-constexpr int kCols2D = 4;          // B: inner-dimension columns per thread, 2D kernel (one float4)
 constexpr int kCols3D = 4;          // B: 3D kernel (one float4)
 constexpr int kMaxPts = 27;
 
@@ -39,20 +38,19 @@ struct HexParams {
 inline int64_t smem_bytes(int ndims, int tT, int tS1, int tS2, int tS3) {
     const int64_t NX = tS1 + tT + 2;
     const int64_t geo = 16 * (int64_t)tT;              // per-level geometry table (ints)
-    if (ndims == 2) return 4 * ((2 * NX + 1) * (tS2 + 4) + 2 * (int64_t)tT * NX * 2 + geo + NX + 2 * (int64_t)tT + 2);
+    if (ndims == 2) return 4 * ((2 * NX + 1) * (tS2 + 8) + 2 * (int64_t)tT * NX * 2 + geo + NX + 2 * (int64_t)tT + 2);
     return 4 * (2 * NX * (tS2 + 2) * (tS3 + 4) + 2 * (int64_t)tT * NX * (tS2 + 2) * 2 + geo);
 }
 
-// 2D column groups per thread (K1): two groups 128 columns apart when tS2 % 256 == 0.
-inline int col_groups_2d(int tS2) { return tS2 % 256 == 0 ? 2 : 1; }
-
+// Column threads of one x-group: 2D K1 threads own 8 columns (4 pairs of the
+// pair layout), 3D K2 threads 4 consecutive tS3 columns of one tS2 line.
 inline int column_threads(int ndims, int tS2, int tS3) {
-    return ndims == 2 ? tS2 / (kCols2D * col_groups_2d(tS2)) : (tS3 / kCols3D) * tS2;
+    return ndims == 2 ? tS2 / 8 : (tS3 / kCols3D) * tS2;
 }
 
 typedef void (*hex_kernel_t)(HexParams);
-hex_kernel_t get_hex_kernel(int ndims, int kind, int mode, bool has_c, bool defw, int ng);
-int hex_kernel_regs(int ndims, int kind, int mode, bool has_c, bool defw, int ng);
+hex_kernel_t get_hex_kernel(int ndims, int kind, int mode, bool has_c, bool defw);
+int hex_kernel_regs(int ndims, int kind, int mode, bool has_c, bool defw);
 void launch_copy_ring(const float* in, float* out, int64_t S1, int64_t S2, int64_t S3, void* stream);
 void launch_copy_full(const float* in, float* out, int64_t n, void* stream);
 

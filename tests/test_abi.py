@@ -53,7 +53,7 @@ def test_create_without_gpu_fails_loudly(lib):
 
 
 def test_tile_validation(lib):
-    assert hhc.stencil_tile_resources(2, (8, 8, 64))[1] == 64        # 16 column threads x 4 groups
+    assert hhc.stencil_tile_resources(2, (8, 8, 64))[1] == 32        # 8 column threads x 4 groups
     for bad in [(7, 8, 64), (0, 8, 64), (8, 0, 64), (8, 8, 48), (8, 8, 0)]:
         with pytest.raises(hhc.StencilError):
             hhc.stencil_tile_resources(2, bad)
@@ -62,7 +62,7 @@ def test_tile_validation(lib):
     with pytest.raises(hhc.StencilError):                              # smem > 227 KB
         hhc.stencil_tile_resources(2, (64, 64, 1024))
     with pytest.raises(hhc.StencilError):                              # threads not a multiple
-        hhc.stencil_tile_resources(2, (8, 8, 64), threads=24)
+        hhc.stencil_tile_resources(2, (8, 8, 64), threads=20)
     sm, thr = hhc.stencil_tile_resources(3, (8, 4, 4, 32))
     assert sm == mo.smem_bytes_exact(3, (8, 4, 4, 32)) and thr == mo.default_threads(3, (8, 4, 4, 32))
 

@@ -264,26 +264,28 @@ def test_virtual_slabs_run_planes(kind, dims, T, tT, nslab):
 
 
 
-NG2_TILES = [((2, 1, 256), 0), ((4, 3, 256), 64), ((8, 5, 512), 0), ((16, 4, 256), 128), ((6, 2, 768), 192),
-             ((10, 7, 1024), 128), ((16, 20, 512), 256), ((12, 9, 256), 32)]
+PAIR_TILES = [((2, 1, 256), 0), ((4, 3, 256), 64), ((8, 5, 512), 0), ((16, 4, 256), 128), ((6, 2, 768), 192),
+              ((10, 7, 1024), 128), ((16, 20, 512), 256), ((12, 9, 256), 32), ((4, 2, 32), 8), ((6, 3, 96), 24),
+              ((8, 6, 160), 80), ((2, 9, 64), 0)]
 
 
 @pytest.mark.parametrize("kind", [hhc.JACOBI2D_5PT, hhc.HEAT2D_9PT, hhc.GRADIENT2D, hhc.LAPLACIAN2D_5PT])
 @pytest.mark.parametrize("mode", [hhc.PLAIN, hhc.FUSED])
-def test_parity_two_column_groups(kind, mode):
-    """K1 with two 4-column groups per thread (tS2 % 256 == 0): random sizes,
-    grids smaller than a tile, odd T, several x-group counts."""
+def test_parity_pair_layout(kind, mode):
+    """K1 pair layout (columns q and q + tS2/2 share a register pair, swizzled
+    chunks): random sizes, grids smaller than a tile, odd T, tS2 from 32 to
+    1024 (non powers of two included), several x-group counts."""
     rng = np.random.default_rng(3000 + kind * 10 + mode)
-    for tile, threads in NG2_TILES:
+    for tile, threads in PAIR_TILES:
         dims = (int(rng.integers(3, 120)), int(rng.integers(3, 1500)))
         a = field(int(rng.integers(1, 1 << 30)), dims)
         for T in (1, 2, 3, tile[0] + 1, 2 * tile[0] + 3):
             exp = oracle.run(kind, a, T, mode)
             got = gpu_run(kind, a, T, tile, mode, threads=threads)
-            assert_bits(got, exp, f"NG2 kind {kind} mode {mode} dims {dims} T {T} tile {tile} thr {threads}")
+            assert_bits(got, exp, f"pair kind {kind} mode {mode} dims {dims} T {T} tile {tile} thr {threads}")
     offs, w = oracle.stencil_info(kind) if kind != hhc.GRADIENT2D else (None, None)
     if w is not None:
         a = field(9, (70, 700))
         coeffs = [float(x) * 0.95 for x in w] + [0.003]
         exp = oracle.run(kind, a, 11, mode, coeffs=coeffs)
-        assert_bits(gpu_run(kind, a, 11, (4, 3, 512), mode, coeffs=coeffs), exp, "NG2 coeffs")
+        assert_bits(gpu_run(kind, a, 11, (4, 3, 512), mode, coeffs=coeffs), exp, "pair coeffs")
