@@ -190,12 +190,12 @@ static int check_tile(int ndims, stencil_tile t, int threads, int smem_limit, in
     }
     if (t.t > 1024 || t.s1 > 4096 || t.s2 > 8192 || (ndims == 3 && t.s3 > 4096)) return STENCIL_ETILE;
     const int base = column_threads(ndims, t.s2, t.s3);
-    if (base > 512) return STENCIL_ETILE;
+    if (base > max_block_threads(ndims)) return STENCIL_ETILE;
     int G;
     if (threads == 0) {
         G = base <= 256 ? std::max(1, std::min(4, 256 / base)) : 1;
     } else {
-        if (threads < 0 || threads > 512 || threads % base) return STENCIL_EINVAL;
+        if (threads < 0 || threads > max_block_threads(ndims) || threads % base) return STENCIL_EINVAL;
         G = threads / base;
     }
     const int64_t sm = smem_bytes(ndims, t.t, t.s1, t.s2, t.s3);
@@ -281,7 +281,7 @@ static int choose_J(stencil_t h, const RowPlan& r) {
 // attribute, its occupancy (for J), and the 3D flag buffer.
 static int prepare_rows(stencil_t h, const int64_t* dims, int64_t T, stencil_tile tile, int thr, int nr = 0) {
     (void)nr;
-    hex_kernel_t k = get_hex_kernel(h->ndims, h->kind, h->mode, h->has_c, h->defw);
+    hex_kernel_t k = get_hex_kernel(h->ndims, h->kind, h->mode, h->has_c, h->defw, tile.s2);
     if (!k) return STENCIL_EINVAL;
     const int64_t smem = smem_bytes(h->ndims, tile.t, tile.s1, tile.s2, tile.s3);
     cudaError_t e = cudaFuncSetAttribute((const void*)k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
@@ -318,7 +318,7 @@ static int enqueue_rows(stencil_t h, const int64_t* dims, const float* ring, flo
     std::vector<RowPlan> rows;
     plan_rows(h->ndims, dims, T, tile, rows);
     (void)nr;
-    hex_kernel_t k = get_hex_kernel(h->ndims, h->kind, h->mode, h->has_c, h->defw);
+    hex_kernel_t k = get_hex_kernel(h->ndims, h->kind, h->mode, h->has_c, h->defw, tile.s2);
     if (!k) return STENCIL_EINVAL;
     const int64_t smem = smem_bytes(h->ndims, tile.t, tile.s1, tile.s2, tile.s3);
     int64_t nl = 0;
@@ -353,6 +353,7 @@ static int enqueue_rows(stencil_t h, const int64_t* dims, const float* ring, flo
     p.kappa = h->kappa;
     p.flags = h->flags;
     p.compute_only = h->compute_only;
+    { static const int dbg = getenv("HHC_DBG") ? atoi(getenv("HHC_DBG")) : 0; p.dbg = dbg; }
     for (auto& r : rows) {
         p.t0 = r.t0; p.xbase = r.xbase; p.tau_lo = r.tau_lo; p.tau_hi = r.tau_hi;
         p.n2 = r.n2; p.n3 = r.n3; p.J = r.J;

@@ -30,6 +30,7 @@ struct HexParams {
     float c;                // Eq. 1 constant
     float kappa;            // Gradient-2D
     int compute_only;       // K4: skip all global<->shared transfers (Citer micro-benchmark)
+    int dbg;                // experiment switches (HHC_DBG, never set in production runs)
 };
 
 // Shared-memory bytes of the HHC kernels (DESIGN.md §Kernels K1/K2): two parity
@@ -44,13 +45,16 @@ inline int64_t smem_bytes(int ndims, int tT, int tS1, int tS2, int tS3) {
 
 // Column threads of one x-group: 2D K1 threads own 8 columns (4 pairs of the
 // pair layout), 3D K2 threads 4 consecutive tS3 columns of one tS2 line.
+// Largest block the HHC kernels launch with (their __launch_bounds__).
+inline int max_block_threads(int ndims) { return ndims == 2 ? 384 : 512; }
+
 inline int column_threads(int ndims, int tS2, int tS3) {
     return ndims == 2 ? tS2 / 8 : (tS3 / kCols3D) * tS2;
 }
 
 typedef void (*hex_kernel_t)(HexParams);
-hex_kernel_t get_hex_kernel(int ndims, int kind, int mode, bool has_c, bool defw);
-int hex_kernel_regs(int ndims, int kind, int mode, bool has_c, bool defw);
+hex_kernel_t get_hex_kernel(int ndims, int kind, int mode, bool has_c, bool defw, int s2);
+int hex_kernel_regs(int ndims, int kind, int mode, bool has_c, bool defw, int s2);
 void launch_copy_ring(const float* in, float* out, int64_t S1, int64_t S2, int64_t S3, void* stream);
 void launch_copy_full(const float* in, float* out, int64_t n, void* stream);
 

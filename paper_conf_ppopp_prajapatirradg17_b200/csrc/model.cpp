@@ -83,7 +83,7 @@ double talg_exact(int nd, const int64_t* S, int64_t T, const stencil_tile& tl, c
     const int64_t Mtile = hhc::smem_bytes(nd, (int)tT, (int)tS1, (int)tS2, (int)tS3);
     const int threads = hw.threads > 0 ? hw.threads : default_threads(nd, tl);
     const int64_t maxthr = hw.max_threads_sm > 0 ? hw.max_threads_sm : 2048;
-    if (Mtile > hw.m_block_bytes || threads > 512) return std::numeric_limits<double>::infinity();
+    if (Mtile > hw.m_block_bytes || threads > hhc::max_block_threads(nd)) return std::numeric_limits<double>::infinity();
     int64_t k = std::min<int64_t>({hw.m_sm_bytes / Mtile, (int64_t)hw.mtb_sm, maxthr / threads});   // Eq. 11
     if (hw.regs_per_thread > 0) k = std::min<int64_t>(k, hw.r_sm / ((int64_t)hw.regs_per_thread * threads));
     if (k < 1) return std::numeric_limits<double>::infinity();

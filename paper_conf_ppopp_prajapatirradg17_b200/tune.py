@@ -130,8 +130,9 @@ def sweep_tiles(nd, limit):
                  for tS3 in (32, 64)]
     out = []
     for t in tiles:
-        base = t[2] // 4 if nd == 2 else (t[3] // 4) * t[2]
-        for threads in sorted({base * g for g in (1, 2, 4, 8) if base * g <= 512}):
+        base = t[2] // 8 if nd == 2 else (t[3] // 4) * t[2]
+        cap = 384 if nd == 2 else 512
+        for threads in sorted({base * g for g in (1, 2, 3, 4, 6, 8) if base * g <= cap}):
             try:
                 hhc.stencil_tile_resources(nd, t, threads)
             except hhc.StencilError:
