@@ -9,9 +9,11 @@ CONFIGS (chosen with model_select_tile + the measured sweep).
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--config C2] [--impl reference]
 
-Under torchrun (N > 1) the same grid is slab-decomposed along S1 across the
-ranks (strong scaling, ghost exchange over NCCL every time tile) and rank 0
-prints the line; times are the max over ranks of device (CUDA-event) time.
+Under torchrun (N > 1) the grid is slab-decomposed along S1 across the ranks
+with a ghost exchange (NCCL P2P) every time tile; by default every rank owns a
+config-sized slab (weak scaling: global grid N*(S1-2)+2 rows), --strong splits
+the config's own grid.  Rank 0 prints the line; times are the max over ranks of
+device (CUDA-event) time.
 """
 from __future__ import annotations
 
@@ -190,6 +192,9 @@ def main(argv=None):
     ap.add_argument("--mode", default="fused", choices=["fused", "plain"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--strong", action="store_true",
+                    help="N > 1: split the config's grid over the ranks (default: weak scaling, one config-sized "
+                         "slab per rank)")
     args = ap.parse_args(argv)
     cfg = CONFIGS[args.config]
     if args.impl == "reference":

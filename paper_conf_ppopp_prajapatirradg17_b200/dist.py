@@ -106,11 +106,15 @@ def run_slabs(slab: Slab, plane0, plane1, T: int, tT: int, stepper, xp_dist):
     return cur
 
 
-def gpu_stepper(handle, tile, threads, stream=None):
+def gpu_stepper(handle, tile, threads, stream=None, counter=None):
+    """Per-tile stepper on the GPU (stencil_run_planes).  `counter`, a one-element
+    list, accumulates the kernel launches the library reports."""
     import paper_conf_ppopp_prajapatirradg17_b200 as hhc
 
     def step(p0, p1, Tt):
         hhc.stencil_run_planes(handle, p0.shape[0], p0, p1, Tt, tile, threads, stream)
+        if counter is not None:
+            counter[0] += hhc.stencil_last_launches(handle)
         return p0 if Tt % 2 == 0 else p1
     return step
 
@@ -135,6 +139,11 @@ def bench_main(args, cfg, cfgname, configs):
     tile = tile + (0,) * (4 - len(tile))
     threads = cfg["threads"] if args.threads is None else args.threads
     dims, T, kind = cfg["dims"], cfg["T"], cfg["kind"]
+    strong = bool(getattr(args, "strong", False))
+    if not strong:
+        # weak scaling (default): every rank owns a slab of the config's interior
+        # rows, the global grid is world times taller; ghost exchange as usual
+        dims = ((dims[0] - 2) * world + 2,) + tuple(dims[1:])
     tT = tile[0]
     slab = partition(dims[0], world, rank, tT)
     ext_dims = (slab.rows,) + tuple(dims[1:])
@@ -144,7 +153,8 @@ def bench_main(args, cfg, cfgname, configs):
     p1 = torch.empty_like(init)
     h = hhc.stencil_create(kind, ext_dims, mode=hhc.FUSED if args.mode == "fused" else hhc.PLAIN)
     stream = torch.cuda.current_stream()
-    step = gpu_stepper(h, tile, threads, stream)
+    launches = [0]
+    step = gpu_stepper(h, tile, threads, stream, launches)
 
     def one():
         p0.copy_(init)
@@ -154,6 +164,12 @@ def bench_main(args, cfg, cfgname, configs):
         one()
     torch.cuda.synchronize()
     dist.barrier()
+    import bench
+    sampler = bench.ClockSampler(local) if rank == 0 else None
+    if sampler:
+        sampler.start()
+        time.sleep(0.3)
+    launches[0] = 0
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     e0.record(stream)
     for _ in range(args.steps):
@@ -161,19 +177,60 @@ def bench_main(args, cfg, cfgname, configs):
     e1.record(stream)
     torch.cuda.synchronize()
     dist.barrier()
-    t = torch.tensor([e0.elapsed_time(e1) * 1e-3], device=dev)
-    dist.all_reduce(t, op=dist.ReduceOp.MAX)
-    dt = float(t.item())
+    clocks = sampler.stop() if sampler else None
+    t = torch.tensor([e0.elapsed_time(e1) * 1e-3, float(launches[0])], device=dev)
+    tmax = t.clone()
+    dist.all_reduce(tmax, op=dist.ReduceOp.MAX)
+    tsum = t.clone()
+    dist.all_reduce(tsum, op=dist.ReduceOp.SUM)
+    dt = float(tmax[0].item())
+    # copies p0 <- init per step (one kernel each) plus the HHC launches of every rank
+    n_launch = int(tsum[1].item()) + world * args.steps
+
+    # e2e through the public API: pinned host slab -> device, the run, owned rows -> host
+    e2e = None
+    if not args.no_e2e:
+        h_in = torch.from_numpy(host).pin_memory()
+        lo, hi = slab.held
+        h_out = torch.empty((hi - lo,) + tuple(dims[1:]), dtype=torch.float32).pin_memory()
+
+        def one_e2e():
+            p0.copy_(h_in, non_blocking=True)
+            out = run_slabs(slab, p0, p1, T, tT, step, dist)
+            h_out.copy_(out[lo - slab.e0:hi - slab.e0], non_blocking=True)
+            torch.cuda.synchronize()
+
+        one_e2e()
+        dist.barrier()
+        t0 = time.perf_counter()
+        for _ in range(args.steps):
+            one_e2e()
+        et = torch.tensor([time.perf_counter() - t0], device=dev)
+        dist.all_reduce(et, op=dist.ReduceOp.MAX)
+        nb = torch.tensor([float(host.nbytes), float(h_out.numel() * 4)], device=dev)
+        dist.all_reduce(nb, op=dist.ReduceOp.SUM)
+        e2e = {"value": hhc.updates(dims, T) * args.steps / float(et.item()) / 1e9, "unit": "GStencil-updates/s",
+               "h2d_bytes_per_step": int(nb[0].item()), "d2h_bytes_per_step": int(nb[1].item())}
     n_upd = hhc.updates(dims, T)
     if rank == 0:
+        flops = bench.FLOPS_PER_UPDATE[kind] * n_upd * args.steps
+        peak = bench.fp32_peak_tflops(bench.load_peaks())
+        ach = flops / dt / world / 1e12
         line = {"metric": "GStencil-updates/s", "value": round(n_upd * args.steps / dt / 1e9, 3),
                 "unit": "GStencil-updates/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
-                "ms_per_step": round(dt / args.steps * 1e3, 3), "higher_is_better": True, "scaling": "strong",
+                "ms_per_step": round(dt / args.steps * 1e3, 3), "higher_is_better": True, "scaling": "strong" if strong else "weak",
                 "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-                "config": {"workload": cfgname + ": " + cfg["desc"], "tile": list(tile), "threads": threads,
+                "config": {"workload": cfgname + ": " + cfg["desc"] + (
+                               "" if strong else f", weak-scaled: {world} slabs of the config's rows, global grid "
+                                                 f"{'x'.join(map(str, dims))}"), "tile": list(tile), "threads": threads,
                            "parallelism": f"{world} S1 slabs, ghost depth {tT}, NCCL P2P every time tile",
                            "l2": "inputs larger than L2"},
-                "gpu_launches": None}
+                "roofline": {"bound": "alu", "achieved": round(ach, 3), "peak": round(peak, 2), "unit": "TFLOP/s",
+                             "frac": round(ach / peak, 4), "traffic": None,
+                             "kernel": "hex2d_kernel" if len(dims) == 2 else "hex3d_kernel",
+                             "basis": "whole-job algorithmic flops / (max-over-ranks step time x n_gpus), "
+                                      "ghost-row redundancy and exchange included"},
+                "e2e": e2e, "clocks": clocks, "gpu_launches": n_launch}
         print(json.dumps(line))
     hhc.stencil_destroy(h)
     dist.destroy_process_group()
