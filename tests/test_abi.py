@@ -153,3 +153,25 @@ def test_select_tile_infeasible(lib):
     c.m_block_bytes = 16
     with pytest.raises(hhc.StencilError):
         hhc.model_select_tile(hhc.HEAT2D_9PT, (66, 66), 10, c)
+
+
+def test_exact_fit_recovers_constants(lib):
+    """tune.fit_exact (reading Q14, EXACT): compute-only times generated as
+    C * A + tau * B are fitted back to (C, tau) (relative least squares)."""
+    import random
+    from paper_conf_ppopp_prajapatirradg17_b200 import tune
+    rnd = random.Random(3)
+    C, tau = 1.3e-8, 2.5e-7
+    insts = []
+    while len(insts) < 25:
+        dims = (rnd.randint(1024, 4096), rnd.randint(1024, 4096))
+        T = rnd.randint(16, 64)
+        tile = tune.random_tile(rnd, 2, dims)
+        a = tune._basis(hhc.HEAT2D_9PT, dims, T, tile, 1.0, 0.0)
+        b = tune._basis(hhc.HEAT2D_9PT, dims, T, tile, 0.0, 1.0)
+        if not (math.isfinite(a) and math.isfinite(b)):
+            continue
+        insts.append((dims, T, tile, (C * a + tau * b) / a))
+    fit = tune.fit_exact(hhc.HEAT2D_9PT, insts)
+    assert abs(fit["C_iter_s"] / C - 1) < 1e-6 and abs(fit["tau_level_s"] / tau - 1) < 1e-6
+    assert fit["rel_rmse"] < 1e-9
