@@ -134,9 +134,10 @@ def cpu_oracle_sample(cfg: dict, seconds: float = 10.0, nthreads: int = 0):
     name = [k for k, v in CONFIGS.items() if v is cfg][0]
     a = field(CONFIG_SEEDS[name], cfg["dims"])
     n_int = math.prod(d - 2 for d in cfg["dims"])
+    oracle.run(cfg["kind"], a, 1, oracle.PLAIN, nthreads=nthreads)        # warm (threads, first touch)
     t0 = time.perf_counter()
-    oracle.run(cfg["kind"], a, 1, oracle.PLAIN, nthreads=nthreads)
-    one = max(time.perf_counter() - t0, 1e-4)
+    oracle.run(cfg["kind"], a, 2, oracle.PLAIN, nthreads=nthreads)
+    one = max((time.perf_counter() - t0) / 2, 1e-4)
     Ts = int(max(1, min(cfg["T"], seconds / one)))
     t0 = time.perf_counter()
     oracle.run(cfg["kind"], a, Ts, oracle.PLAIN, nthreads=nthreads)
