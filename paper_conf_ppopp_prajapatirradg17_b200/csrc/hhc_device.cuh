@@ -223,6 +223,24 @@ __device__ __forceinline__ void cp_async4(float* dst, const float* src) {
 }
 __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;\n" ::: "memory"); }
 
+// Four consecutive floats src[0..3] -> dst[0..3] (dst 16-B aligned) with the
+// widest cp.async the source alignment allows (16, 8 or 4 bytes per copy); the
+// skew makes the source alignment level-dependent (3D footprint lines).
+__device__ __forceinline__ void cp_async_f4(float* dst, const float* src) {
+    const unsigned s = (unsigned)__cvta_generic_to_shared(dst);
+    const unsigned a = (unsigned)(uintptr_t)src & 15u;
+    if (a == 0) {
+        asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(s), "l"(src) : "memory");
+    } else if ((a & 7u) == 0) {
+        asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(s), "l"(src) : "memory");
+        asm volatile("cp.async.ca.shared.global [%0], [%1], 8;\n" ::"r"(s + 8), "l"(src + 2) : "memory");
+    } else {
+#pragma unroll
+        for (int j = 0; j < 4; ++j)
+            asm volatile("cp.async.ca.shared.global [%0], [%1], 4;\n" ::"r"(s + 4 * j), "l"(src + j) : "memory");
+    }
+}
+
 // Non-facet interval [lo, hi) of smem rows at one level (reading G3): rows whose
 // every reader at the next level lies inside this block.  Empty -> write all.
 __device__ __forceinline__ void facet_gap(int64_t nl, int64_t nr, int64_t S1, bool final_level, int64_t xs,
