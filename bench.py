@@ -35,7 +35,7 @@ CONFIGS = {
                desc="Heat-2D 9-point fp32, 8192x8192, T=1024"),
     "C3": dict(kind=3, dims=(16384, 16384), T=512, tile=(32, 12, 512, 0), threads=384,
                desc="Gradient-2D fp32, 16384x16384, T=512"),
-    "C4": dict(kind=4, dims=(512, 512, 512), T=256, tile=(10, 8, 8, 64), threads=512,
+    "C4": dict(kind=4, dims=(512, 512, 512), T=256, tile=(8, 8, 16, 64), threads=512,
                desc="Heat-3D 7-point fp32, 512^3, T=256"),
     "C5": dict(kind=5, dims=(768, 768, 768), T=128, tile=(8, 6, 8, 64), threads=256,
                desc="Laplacian-3D 27-point fp32, 768^3, T=128"),
