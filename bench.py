@@ -193,6 +193,8 @@ def main(argv=None):
     ap.add_argument("--mode", default="fused", choices=["fused", "plain"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-overlap", action="store_true",
+                    help="N>1: exchange, then the whole ghost-extended slab (no overlap)")
     ap.add_argument("--strong", action="store_true",
                     help="N > 1: split the config's grid over the ranks (default: weak scaling, one config-sized "
                          "slab per rank)")

@@ -106,6 +106,99 @@ def run_slabs(slab: Slab, plane0, plane1, T: int, tT: int, stepper, xp_dist):
     return cur
 
 
+def run_slabs_overlap(slab: Slab, plane0, plane1, T: int, tT: int, stepper_int, stepper_edge, xp_dist,
+                      streams=None):
+    """The time-tile loop with the exchange overlapped (SURVEY §8(e) "Overlap").
+
+    Per tile: the two edge sub-slabs -- 3g rows around each neighbour side, fresh
+    ghosts included -- run first (stepper_edge, second stream) and their exact
+    owned rows [lo, lo+g) / [hi-g, hi) are sent to the neighbours at once; the
+    interior sub-slab (the owned rows alone, whose edge rows act as a fixed ring
+    for the tile) needs no ghosts and runs concurrently (stepper_int, first
+    stream).  After tT <= g steps the interior run is exact on [lo+g, hi-g), the
+    edge runs on the g rows next to each side (dependence cone of tT rows), so
+    the tile's result is the interior plane with the edge rows and the received
+    ghosts written in.  Redundant work: 3g rows per neighbour side per tile.
+
+    `streams` = (s1, s2) torch.cuda streams, or None (CPU: sequential).  Falls
+    back to run_slabs when a slab is thinner than 2g rows."""
+    import torch
+    g = slab.g
+    lo, hi = slab.r0 - slab.e0, slab.r1 - slab.e0
+    up, dn = slab.rank > 0, slab.rank < slab.world - 1
+    if not (up or dn) or hi - lo < 2 * g:
+        return run_slabs(slab, plane0, plane1, T, tT, stepper_int, xp_dist)
+    A, B = (lo if up else 0), (hi if dn else slab.rows)
+    tail = tuple(plane0.shape[1:])
+
+    def buf(n):
+        return torch.empty((n,) + tail, dtype=plane0.dtype, device=plane0.device)
+
+    e_up = (lo - g, lo + 2 * g) if up else None          # local rows of the edge sub-slabs
+    e_dn = (hi - 2 * g, hi + g) if dn else None
+    t_bufs = (buf(3 * g), buf(3 * g)) if up else None
+    b_bufs = (buf(3 * g), buf(3 * g)) if dn else None
+    r_up = buf(g) if up else None
+    r_dn = buf(g) if dn else None
+    s1, s2 = streams if streams is not None else (None, None)
+
+    def on(st):
+        return torch.cuda.stream(st) if st is not None else _Null()
+
+    exchange(slab, plane0, xp_dist)                      # ghosts of tile 0 (blocking)
+    cur, oth = plane0, plane1
+    done = 0
+    while done < T:
+        Tt = min(tT, T - done)
+        last = done + Tt >= T
+        with on(s1):                                     # edge inputs taken before the interior overwrites cur
+            if up:
+                t_bufs[0].copy_(cur[e_up[0]:e_up[1]])
+            if dn:
+                b_bufs[0].copy_(cur[e_dn[0]:e_dn[1]])
+        if s2 is not None:
+            s2.wait_stream(s1)
+        works = []
+        with on(s2):
+            te = stepper_edge(t_bufs[0], t_bufs[1], Tt) if up else None
+            be = stepper_edge(b_bufs[0], b_bufs[1], Tt) if dn else None
+            if not last:
+                ops = []
+                if up:
+                    ops.append(xp_dist.P2POp(xp_dist.isend, te[g:2 * g], slab.rank - 1))
+                    ops.append(xp_dist.P2POp(xp_dist.irecv, r_up, slab.rank - 1))
+                if dn:
+                    ops.append(xp_dist.P2POp(xp_dist.isend, be[g:2 * g], slab.rank + 1))
+                    ops.append(xp_dist.P2POp(xp_dist.irecv, r_dn, slab.rank + 1))
+                works = xp_dist.batch_isend_irecv(ops)
+        with on(s1):
+            stepper_int(cur[A:B], oth[A:B], Tt)           # overlaps the exchange
+            res = cur if Tt % 2 == 0 else oth
+            if s2 is not None:
+                s1.wait_stream(s2)
+            for w in works:
+                w.wait()
+            if up:
+                res[lo:lo + g].copy_(te[g:2 * g])
+                if not last:
+                    res[lo - g:lo].copy_(r_up)
+            if dn:
+                res[hi - g:hi].copy_(be[g:2 * g])
+                if not last:
+                    res[hi:hi + g].copy_(r_dn)
+        cur, oth = res, (plane1 if res is plane0 else plane0)
+        done += Tt
+    return cur
+
+
+class _Null:
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        return False
+
+
 def gpu_stepper(handle, tile, threads, stream=None, counter=None):
     """Per-tile stepper on the GPU (stencil_run_planes).  `counter`, a one-element
     list, accumulates the kernel launches the library reports."""
@@ -151,14 +244,26 @@ def bench_main(args, cfg, cfgname, configs):
     init = torch.from_numpy(host).to(dev)
     p0 = torch.empty_like(init)
     p1 = torch.empty_like(init)
-    h = hhc.stencil_create(kind, ext_dims, mode=hhc.FUSED if args.mode == "fused" else hhc.PLAIN)
+    mode = hhc.FUSED if args.mode == "fused" else hhc.PLAIN
+    h = hhc.stencil_create(kind, ext_dims, mode=mode)
     stream = torch.cuda.current_stream()
     launches = [0]
     step = gpu_stepper(h, tile, threads, stream, launches)
+    overlap = not getattr(args, "no_overlap", False)
+    if overlap:
+        # edge sub-slabs on a second stream with their own handle (3D progress flags)
+        side = torch.cuda.Stream(device=dev)
+        h_edge = hhc.stencil_create(kind, ext_dims, mode=mode)
+        step_edge = gpu_stepper(h_edge, tile, threads, side, launches)
+
+    def drive(a, b):
+        if overlap:
+            return run_slabs_overlap(slab, a, b, T, tT, step, step_edge, dist, (stream, side))
+        return run_slabs(slab, a, b, T, tT, step, dist)
 
     def one():
         p0.copy_(init)
-        return run_slabs(slab, p0, p1, T, tT, step, dist)
+        return drive(p0, p1)
 
     for _ in range(args.warmup):
         one()
@@ -196,7 +301,7 @@ def bench_main(args, cfg, cfgname, configs):
 
         def one_e2e():
             p0.copy_(h_in, non_blocking=True)
-            out = run_slabs(slab, p0, p1, T, tT, step, dist)
+            out = drive(p0, p1)
             h_out.copy_(out[lo - slab.e0:hi - slab.e0], non_blocking=True)
             torch.cuda.synchronize()
 
@@ -223,7 +328,9 @@ def bench_main(args, cfg, cfgname, configs):
                 "config": {"workload": cfgname + ": " + cfg["desc"] + (
                                "" if strong else f", weak-scaled: {world} slabs of the config's rows, global grid "
                                                  f"{'x'.join(map(str, dims))}"), "tile": list(tile), "threads": threads,
-                           "parallelism": f"{world} S1 slabs, ghost depth {tT}, NCCL P2P every time tile",
+                           "parallelism": f"{world} S1 slabs, ghost depth {tT}, NCCL P2P every time tile"
+                                          + (", exchange overlapped with the interior sub-slab (edge sub-slabs "
+                                             "first on a second stream)" if overlap else ""),
                            "l2": "inputs larger than L2"},
                 "roofline": {"bound": "alu", "achieved": round(ach, 3), "peak": round(peak, 2), "unit": "TFLOP/s",
                              "frac": round(ach / peak, 4), "traffic": None,
@@ -233,5 +340,7 @@ def bench_main(args, cfg, cfgname, configs):
                 "e2e": e2e, "clocks": clocks, "gpu_launches": n_launch}
         print(json.dumps(line))
     hhc.stencil_destroy(h)
+    if overlap:
+        hhc.stencil_destroy(h_edge)
     dist.destroy_process_group()
     return 0
