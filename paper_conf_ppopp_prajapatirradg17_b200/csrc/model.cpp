@@ -122,12 +122,17 @@ double talg_exact(int nd, const int64_t* S, int64_t T, const stencil_tile& tl, c
             csum += (double)cdiv(W * inner, hw.n_v);           // Eq. 15 / 27, row by row
         }
         double Nsub, mi, mo, extra = 0.0;
+        int64_t J = 1;
         if (nd == 2) {
             Nsub = (double)cdiv(S2 + nlev - 1, tS2);
             mi = (double)reads * (double)(tS2 + 2);
             mo = (double)writes * (double)tS2;
         } else {
-            Nsub = (double)(cdiv(S2 + nlev - 1, tS2) * cdiv(S3 + nlev - 1, tS3));
+            // reading M8: J blocks per slab pipelined along S2 (the library's choice);
+            // a block sweeps ceil(n2/J)*n3 sub-slabs, the last starts J-1 sub-slabs late
+            const int64_t n2 = cdiv(S2 + nlev - 1, tS2), n3 = cdiv(S3 + nlev - 1, tS3);
+            J = std::max<int64_t>(1, std::min<int64_t>(n2, ((int64_t)hw.n_sm * k) / w));
+            Nsub = (double)(cdiv(n2, J) * n3 + (J - 1));
             mi = (double)reads * (double)((tS2 + 2) * (tS3 + 2));
             mo = (double)writes * (double)(tS2 * tS3);
             extra = 4.0 * (double)tS3 * (double)area;           // S2 face through global memory
@@ -137,7 +142,7 @@ double talg_exact(int nd, const int64_t* S, int64_t T, const stencil_tile& tl, c
         double Tprism;
         if (k == 1) Tprism = (m_prime + c) * Nsub;                                 // Eq. 16 / 28
         else Tprism = m_prime + (double)k * std::max(m_prime, c) * Nsub;           // Eq. 16 / 29
-        const double v = Tprism * (double)cdiv(cdiv(w, k), hw.n_sm);              // Eq. 2
+        const double v = Tprism * (double)cdiv(cdiv(w * J, k), hw.n_sm);          // Eq. 2
         key_prev[ph] = key;
         val_prev[ph] = v;
         total += v;

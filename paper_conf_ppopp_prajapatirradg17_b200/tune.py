@@ -93,7 +93,7 @@ def calibrate(args):
     out["tau_sync_s"] = hhc.stencil_microbench(1, threads=256)
     out["T_sync_s"] = hhc.stencil_microbench(2)
     rnd = random.Random(2017)
-    citer, samples, fits, insts = {}, {}, {}, []
+    citer, samples, fits, insts, raw = {}, {}, {}, [], {}
     for kind in KINDS:
         nd = hhc.KIND_NDIMS[kind]
         vals = []
@@ -116,16 +116,18 @@ def calibrate(args):
         citer[str(kind)] = sum(vals) / len(vals)
         samples[str(kind)] = {"n": len(vals), "min": min(vals), "max": max(vals)}
         fits[str(kind)] = fit_exact(kind, insts)
+        raw[str(kind)] = [[list(d), T_, list(t), v] for d, T_, t, v in insts]
         insts.clear()
         print(f"C_iter kind {kind}: {citer[str(kind)]:.3e} s over {len(vals)} instances; "
               f"EXACT fit {fits[str(kind)]}", flush=True)
     out["C_iter_s"] = citer
     out["C_iter_samples"] = samples
     out["exact_fit"] = fits
+    out["instances"] = raw          # (dims, T, tile, compute-only seconds): refits need no GPU
     os.makedirs(os.path.dirname(args.out), exist_ok=True)
     with open(args.out, "w") as f:
         json.dump(out, f, indent=1)
-    print(json.dumps({k: v for k, v in out.items() if k != "C_iter_samples"}))
+    print(json.dumps({k: v for k, v in out.items() if k not in ("C_iter_samples", "instances")}))
 
 
 def _basis(kind, dims, T, tile, c_iter, tau):
