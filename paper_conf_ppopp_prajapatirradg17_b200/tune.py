@@ -173,7 +173,7 @@ def sweep_tiles(nd, limit):
         tiles = [(tT, tS1, tS2, 0) for tT in (4, 8, 12, 16, 24, 32) for tS1 in (4, 8, 12, 16, 20, 28)
                  for tS2 in (128, 256, 512)]
     else:
-        tiles = [(tT, tS1, tS2, tS3) for tT in (2, 4, 8) for tS1 in (2, 4, 8) for tS2 in (2, 4, 8)
+        tiles = [(tT, tS1, tS2, tS3) for tT in (2, 4, 6, 8, 10) for tS1 in (2, 4, 6, 8) for tS2 in (2, 4, 8, 16)
                  for tS3 in (32, 64)]
     out = []
     for t in tiles:
