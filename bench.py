@@ -39,13 +39,16 @@ CONFIGS = {
                desc="Heat-3D 7-point fp32, 512^3, T=256"),
     "C5": dict(kind=5, dims=(768, 768, 768), T=128, tile=(8, 6, 8, 64), threads=256,
                desc="Laplacian-3D 27-point fp32, 768^3, T=128"),
+    # SURVEY §8(f) f2 (not a BASELINE.json config): the paper's 1D derivation case
+    "X1": dict(kind=7, dims=(1 << 26,), T=1024, tile=(64, 2048), threads=256,
+               desc="Jacobi-1D 3-point fp32, 2^26 points, T=1024 (extension f2)"),
 }
 DEFAULT_CONFIG = "C2"
 
 # Algorithmic FP32 flops per update of the canonical fused expression
 # (DESIGN.md §Roofline): linear kinds 1 mul + (|N|-1) fma = 2|N|-1; Gradient
 # 19 (sqrt and div counted as one flop each, their SASS sequences are longer).
-FLOPS_PER_UPDATE = {1: 9, 2: 17, 3: 19, 4: 13, 5: 53, 6: 9}
+FLOPS_PER_UPDATE = {1: 9, 2: 17, 3: 19, 4: 13, 5: 53, 6: 9, 7: 5}
 
 METRIC = "GStencil-updates/s"
 
@@ -142,6 +145,11 @@ def cpu_oracle_sample(cfg: dict, seconds: float = 10.0, nthreads: int = 0):
     t0 = time.perf_counter()
     oracle.run(cfg["kind"], a, Ts, oracle.PLAIN, nthreads=nthreads)
     dt = time.perf_counter() - t0
+    if dt < 0.5 * seconds and Ts < cfg["T"]:           # the 2-step estimate was pessimistic: resize once
+        Ts = int(max(1, min(cfg["T"], Ts * seconds / max(dt, 1e-3))))
+        t0 = time.perf_counter()
+        oracle.run(cfg["kind"], a, Ts, oracle.PLAIN, nthreads=nthreads)
+        dt = time.perf_counter() - t0
     cores = nthreads or oracle.max_threads()
     return {"value": n_int * Ts / dt / 1e9, "unit": METRIC, "cores": cores, "kind": "oracle",
             "sample": f"full {'x'.join(map(str, cfg['dims']))} grid, {Ts} of {cfg['T']} steps, plain mode, "
@@ -262,7 +270,7 @@ def bench_single(args, cfg, cfgname):
     traffic = ncu_traffic(cfgname)
     roofline = {"bound": "alu", "achieved": round(achieved, 3), "peak": round(peak, 2), "unit": "TFLOP/s",
                 "frac": round(achieved / peak, 4), "traffic": traffic,
-                "kernel": "hex2d_kernel" if len(dims) == 2 else "hex3d_kernel",
+                "kernel": {1: "hex1d_kernel", 2: "hex2d_kernel", 3: "hex3d_kernel"}[len(dims)],
                 "kernel_share_of_step": round(ksec / (dt / args.steps), 4),
                 "kernel_launches_per_step": klaunch,
                 "peak_basis": "148 SM x 128 FP32 lanes x 2 x sm_max_mhz (MEASURED_PEAKS.json)"}

@@ -45,7 +45,9 @@ typedef enum {
     STENCIL_GRADIENT2D = 3,        /* non-linear 5-point, kappa = 1/8                       */
     STENCIL_HEAT3D_7PT = 4,        /* centre + 6 faces, 1/4, 1/8                            */
     STENCIL_LAPLACIAN3D_27PT = 5,  /* 3x3x3 box, 1/2, 7/128, 3/256, 1/256                   */
-    STENCIL_LAPLACIAN2D_5PT = 6    /* centre + 4 faces, 1/2, 1/8                            */
+    STENCIL_LAPLACIAN2D_5PT = 6,   /* centre + 4 faces, 1/2, 1/8                            */
+    STENCIL_JACOBI1D_3PT = 7       /* 1D: x-1, x, x+1, weights fp32(1/3) (the
+                                      paper's Section 4.1 derivation)           */
 } stencil_kind;
 
 typedef enum {
@@ -90,7 +92,8 @@ typedef struct {
 typedef struct stencil_s* stencil_t;     /* opaque; owned by the library */
 
 /* Create a handle for one stencil problem on the CURRENT CUDA device.
- *   kind/ndims must agree (2D kinds: ndims = 2; 3D kinds: ndims = 3);
+ *   kind/ndims must agree (1D kind: ndims = 1; 2D kinds: ndims = 2; 3D kinds: ndims = 3);
+ *   1D tiles are (t, s1, 0, 0): hexagons of base s1 (>= 1) and height t, 256 threads;
  *   dims[ndims] are full extents, each >= 3;
  *   coeffs == NULL -> the default weights of DESIGN.md R1.  Linear kinds take
  *   |N| weights in canonical (lexicographic offset) order, optionally followed

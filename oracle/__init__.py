@@ -27,7 +27,8 @@ _SRC = os.path.join(_HERE, "stencil_oracle.c")
 _LIB = os.path.join(_HERE, "liboracle.so")
 
 JACOBI2D_5PT, HEAT2D_9PT, GRADIENT2D, HEAT3D_7PT, LAPLACIAN3D_27PT, LAPLACIAN2D_5PT = 1, 2, 3, 4, 5, 6
-KIND_NDIMS = {1: 2, 2: 2, 3: 2, 4: 3, 5: 3, 6: 2}
+JACOBI1D_3PT = 7
+KIND_NDIMS = {1: 2, 2: 2, 3: 2, 4: 3, 5: 3, 6: 2, 7: 1}
 PLAIN, FUSED = 0, 1
 
 CFLAGS = ["-O2", "-ffp-contract=off", "-fno-fast-math", "-fopenmp", "-shared", "-fPIC"]

@@ -31,7 +31,7 @@
 /* Stencil kinds (numbering is part of the C ABI contract in include/hhc.h,
  * re-declared here on purpose: the oracle includes nothing from the product). */
 enum { O_JACOBI2D_5PT = 1, O_HEAT2D_9PT = 2, O_GRADIENT2D = 3,
-       O_HEAT3D_7PT = 4, O_LAPLACIAN3D_27PT = 5, O_LAPLACIAN2D_5PT = 6 };
+       O_HEAT3D_7PT = 4, O_LAPLACIAN3D_27PT = 5, O_LAPLACIAN2D_5PT = 6, O_JACOBI1D_3PT = 7 };
 enum { O_MODE_PLAIN = 0, O_MODE_FUSED = 1 };
 
 typedef struct {
@@ -49,6 +49,7 @@ static int o_kind_ndims(int kind) {
     switch (kind) {
     case O_JACOBI2D_5PT: case O_HEAT2D_9PT: case O_GRADIENT2D: case O_LAPLACIAN2D_5PT: return 2;
     case O_HEAT3D_7PT: case O_LAPLACIAN3D_27PT: return 3;
+    case O_JACOBI1D_3PT: return 1;
     default: return 0;
     }
 }
@@ -58,7 +59,7 @@ static int o_in_neigh(int kind, int nz) {
     switch (kind) {
     case O_JACOBI2D_5PT: case O_LAPLACIAN2D_5PT: case O_HEAT3D_7PT: case O_GRADIENT2D:
         return nz <= 1;                        /* centre + faces */
-    case O_HEAT2D_9PT: case O_LAPLACIAN3D_27PT:
+    case O_HEAT2D_9PT: case O_LAPLACIAN3D_27PT: case O_JACOBI1D_3PT:
         return 1;                              /* full 3^D box */
     default: return 0;
     }
@@ -69,6 +70,7 @@ static int o_in_neigh(int kind, int nz) {
 static float o_default_weight(int kind, int nz) {
     switch (kind) {
     case O_JACOBI2D_5PT: return 0.2f;
+    case O_JACOBI1D_3PT: return 1.0f / 3.0f;   /* PolyBench jacobi-1d averaging, fp32(1/3) */
     case O_LAPLACIAN2D_5PT: return nz == 0 ? 0.5f : 0.125f;
     case O_HEAT2D_9PT: return nz == 0 ? 0.25f : (nz == 1 ? 0.125f : 0.0625f);
     case O_HEAT3D_7PT: return nz == 0 ? 0.25f : 0.125f;
@@ -93,8 +95,9 @@ static int o_build(int kind, const float* coeffs, int ncoeffs, o_stencil* s) {
     }
     int D = s->ndims;
     int lo3 = (D == 3) ? -1 : 0, hi3 = (D == 3) ? 1 : 0;
+    int lo2 = (D >= 2) ? -1 : 0, hi2 = (D >= 2) ? 1 : 0;
     for (int d1 = -1; d1 <= 1; ++d1)
-        for (int d2 = -1; d2 <= 1; ++d2)
+        for (int d2 = lo2; d2 <= hi2; ++d2)
             for (int d3 = lo3; d3 <= hi3; ++d3) {
                 int nz = (d1 != 0) + (d2 != 0) + (d3 != 0);
                 if (!o_in_neigh(kind, nz)) continue;
@@ -153,11 +156,12 @@ int oracle_run(int kind, int ndims, const int64_t* dims, const float* coeffs, in
     if (o_build(kind, coeffs, ncoeffs, &s) != 0) return -1;
     if (ndims != s.ndims || T < 0 || !in || !out) return -1;
     if (mode != O_MODE_PLAIN && mode != O_MODE_FUSED) return -1;
-    int64_t S1 = dims[0], S2 = dims[1], S3 = (ndims == 3) ? dims[2] : 1;
-    if (S1 < 3 || S2 < 3 || (ndims == 3 && S3 < 3)) return -1;
+    int64_t S1 = dims[0], S2 = (ndims >= 2) ? dims[1] : 1, S3 = (ndims == 3) ? dims[2] : 1;
+    if (S1 < 3 || (ndims >= 2 && S2 < 3) || (ndims == 3 && S3 < 3)) return -1;
     int64_t n = S1 * S2 * S3;
     int64_t stride[3] = { S2 * S3, S3, 1 };
     if (ndims == 2) { stride[0] = S2; stride[1] = 1; stride[2] = 0; }
+    if (ndims == 1) { stride[0] = 1; stride[1] = 0; stride[2] = 0; }
     float* plane[2];
     plane[0] = out;
     plane[1] = (float*)malloc((size_t)n * sizeof(float));
@@ -168,7 +172,10 @@ int oracle_run(int kind, int ndims, const int64_t* dims, const float* coeffs, in
     for (int64_t t = 1; t <= T; ++t) {
         const float* src = plane[(t - 1) & 1];
         float* dst = plane[t & 1];
-        if (ndims == 2) {
+        if (ndims == 1) {
+            #pragma omp parallel for num_threads(nt) schedule(static)
+            for (int64_t x = 1; x < S1 - 1; ++x) dst[x] = o_point_linear(&s, src, x, stride, mode);
+        } else if (ndims == 2) {
             #pragma omp parallel for num_threads(nt) schedule(static)
             for (int64_t x = 1; x < S1 - 1; ++x)
                 for (int64_t y = 1; y < S2 - 1; ++y) {

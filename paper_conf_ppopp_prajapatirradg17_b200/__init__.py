@@ -20,9 +20,10 @@ LIB_PATH = os.path.join(_HERE, "libhhc.so")
 
 # stencil_kind (include/hhc.h)
 JACOBI2D_5PT, HEAT2D_9PT, GRADIENT2D, HEAT3D_7PT, LAPLACIAN3D_27PT, LAPLACIAN2D_5PT = 1, 2, 3, 4, 5, 6
+JACOBI1D_3PT = 7          # the paper's 1D derivation case
 KIND_NAMES = {1: "Jacobi-2D 5-point", 2: "Heat-2D 9-point", 3: "Gradient-2D", 4: "Heat-3D 7-point",
               5: "Laplacian-3D 27-point", 6: "Laplacian-2D 5-point"}
-KIND_NDIMS = {1: 2, 2: 2, 3: 2, 4: 3, 5: 3, 6: 2}
+KIND_NDIMS = {1: 2, 2: 2, 3: 2, 4: 3, 5: 3, 6: 2, 7: 1}
 PLAIN, FUSED = 0, 1
 PAPER, EXACT = 0, 1
 

@@ -20,6 +20,7 @@ int kind_ndims_host(int kind) {
     case STENCIL_JACOBI2D_5PT: case STENCIL_HEAT2D_9PT: case STENCIL_GRADIENT2D:
     case STENCIL_LAPLACIAN2D_5PT: return 2;
     case STENCIL_HEAT3D_7PT: case STENCIL_LAPLACIAN3D_27PT: return 3;
+    case STENCIL_JACOBI1D_3PT: return 1;
     default: return 0;
     }
 }
@@ -28,6 +29,7 @@ int kind_ndims_host(int kind) {
 float default_weight(int kind, int nz) {
     switch (kind) {
     case STENCIL_JACOBI2D_5PT: return 0.2f;
+    case STENCIL_JACOBI1D_3PT: return 1.0f / 3.0f;
     case STENCIL_LAPLACIAN2D_5PT: return nz == 0 ? 0.5f : 0.125f;
     case STENCIL_HEAT2D_9PT: return nz == 0 ? 0.25f : (nz == 1 ? 0.125f : 0.0625f);
     case STENCIL_HEAT3D_7PT: return nz == 0 ? 0.25f : 0.125f;
@@ -38,7 +40,8 @@ float default_weight(int kind, int nz) {
 }
 
 bool in_nb(int kind, int nz) {
-    return (kind == STENCIL_HEAT2D_9PT || kind == STENCIL_LAPLACIAN3D_27PT) ? true : nz <= 1;
+    return (kind == STENCIL_HEAT2D_9PT || kind == STENCIL_LAPLACIAN3D_27PT || kind == STENCIL_JACOBI1D_3PT) ? true
+                                                                                                           : nz <= 1;
 }
 
 
@@ -145,7 +148,7 @@ extern "C" int stencil_create(stencil_kind kind, int ndims, const int64_t* dims,
     } else {
         int n = 0;
         for (int d1 = -1; d1 <= 1; ++d1)
-            for (int d2 = -1; d2 <= 1; ++d2)
+            for (int d2 = (D >= 2 ? -1 : 0); d2 <= (D >= 2 ? 1 : 0); ++d2)
                 for (int d3 = (D == 3 ? -1 : 0); d3 <= (D == 3 ? 1 : 0); ++d3) {
                     const int nz = (d1 != 0) + (d2 != 0) + (d3 != 0);
                     if (!in_nb(kind, nz)) continue;
@@ -183,6 +186,15 @@ extern "C" void stencil_destroy(stencil_t h) {
 // ---- tile validation (§8(b) validation rules; Eq. 31 integrality)
 static int check_tile(int ndims, stencil_tile t, int threads, int smem_limit, int* G_out, int* thr_out) {
     if (t.t < 2 || (t.t & 1) || t.s1 < 1) return STENCIL_ETILE;
+    if (ndims == 1) {
+        if (t.t > 1024 || t.s1 > 65536) return STENCIL_ETILE;
+        if (threads != 0 && threads != 256) return STENCIL_EINVAL;
+        const int64_t sm = smem_bytes(1, t.t, t.s1, 0, 0);
+        if (sm > smem_limit) return STENCIL_ETILE;
+        *G_out = 1;
+        *thr_out = 256;
+        return STENCIL_OK;
+    }
     if (ndims == 2) {
         if (t.s2 < 32 || t.s2 % 32) return STENCIL_ETILE;
     } else {
@@ -207,7 +219,7 @@ static int check_tile(int ndims, stencil_tile t, int threads, int smem_limit, in
 
 extern "C" int stencil_tile_resources(int ndims, stencil_tile tile, int threads, int64_t* smem,
                                       int* block_threads, int* regs) {
-    if (ndims != 2 && ndims != 3) return STENCIL_EINVAL;
+    if (ndims < 1 || ndims > 3) return STENCIL_EINVAL;
     int G, thr;
     const int rc = check_tile(ndims, tile, threads, 227 * 1024, &G, &thr);
     if (rc) return rc;
@@ -236,7 +248,10 @@ static void plan_rows(int ndims, const int64_t* dims, int64_t T, stencil_tile t,
         r.xbase = A ? 1 : 1 + t.s1 + h;
         r.w = (int)(A ? wA : wB);
         const int nlev = r.tau_hi - r.tau_lo;
-        if (ndims == 2) {
+        if (ndims == 1) {
+            r.n2 = 1;
+            r.n3 = 1;
+        } else if (ndims == 2) {
             r.n2 = (int)cdiv(dims[1] - 2 + nlev - 1, t.s2);
             r.n3 = 1;
         } else {
@@ -250,7 +265,7 @@ static void plan_rows(int ndims, const int64_t* dims, int64_t T, stencil_tile t,
 
 extern "C" int stencil_plan_info(int ndims, const int64_t* dims, int64_t T, stencil_tile tile,
                                  int64_t* n_rows, int64_t* w_a, int64_t* w_b, int64_t* n_sub) {
-    if ((ndims != 2 && ndims != 3) || !dims || T < 1) return STENCIL_EINVAL;
+    if (ndims < 1 || ndims > 3 || !dims || T < 1) return STENCIL_EINVAL;
     int G, thr;
     const int rc = check_tile(ndims, tile, 0, 1 << 30, &G, &thr);
     if (rc) return rc;
@@ -343,7 +358,7 @@ static int enqueue_rows(stencil_t h, const int64_t* dims, const float* ring, flo
     p.in = ring;
     p.plane[0] = plane0;
     p.plane[1] = plane1;
-    p.S1 = dims[0]; p.S2 = dims[1]; p.S3 = h->ndims == 3 ? dims[2] : 1;
+    p.S1 = dims[0]; p.S2 = h->ndims >= 2 ? dims[1] : 1; p.S3 = h->ndims == 3 ? dims[2] : 1;
     p.T = T;
     p.tT = tile.t; p.tS1 = tile.s1; p.tS2 = tile.s2; p.tS3 = h->ndims == 3 ? tile.s3 : 0;
     p.G = G;

@@ -39,6 +39,7 @@ struct HexParams {
 inline int64_t smem_bytes(int ndims, int tT, int tS1, int tS2, int tS3) {
     const int64_t NX = tS1 + tT + 2;
     const int64_t geo = 16 * (int64_t)tT;              // per-level geometry table (ints)
+    if (ndims == 1) return 4 * (2 * NX + geo);         // K0: two planes of NX values + geometry
     if (ndims == 2) return 4 * ((2 * NX + 1) * (tS2 + 8) + 2 * (int64_t)tT * NX * 2 + geo + NX + 2 * (int64_t)tT + 2 + 2 * NX);
     return 4 * (2 * NX * (tS2 + 2) * (tS3 + 4) + 2 * (int64_t)tT * NX * (tS2 + 2) * 2 + geo);
 }
@@ -46,10 +47,10 @@ inline int64_t smem_bytes(int ndims, int tT, int tS1, int tS2, int tS3) {
 // Column threads of one x-group: 2D K1 threads own 8 columns (4 pairs of the
 // pair layout), 3D K2 threads 4 consecutive tS3 columns of one tS2 line.
 // Largest block the HHC kernels launch with (their __launch_bounds__).
-inline int max_block_threads(int ndims) { return ndims == 2 ? 384 : 512; }
+inline int max_block_threads(int ndims) { return ndims == 1 ? 256 : ndims == 2 ? 384 : 512; }
 
 inline int column_threads(int ndims, int tS2, int tS3) {
-    return ndims == 2 ? tS2 / 8 : (tS3 / kCols3D) * tS2;
+    return ndims == 1 ? 256 : ndims == 2 ? tS2 / 8 : (tS3 / kCols3D) * tS2;
 }
 
 typedef void (*hex_kernel_t)(HexParams);

@@ -22,18 +22,41 @@ int ndims_of(int kind) {
     case STENCIL_JACOBI2D_5PT: case STENCIL_HEAT2D_9PT: case STENCIL_GRADIENT2D:
     case STENCIL_LAPLACIAN2D_5PT: return 2;
     case STENCIL_HEAT3D_7PT: case STENCIL_LAPLACIAN3D_27PT: return 3;
+    case STENCIL_JACOBI1D_3PT: return 1;
     default: return 0;
     }
 }
 
 bool tile_ok(int nd, const stencil_tile& t) {
+    if (nd == 1) return t.t >= 2 && !(t.t & 1) && t.s1 >= 1;
     if (t.t < 2 || (t.t & 1) || t.s1 < 1 || t.s2 < 1) return false;
     if (nd == 2) return t.s2 % 32 == 0;
     return t.s3 >= 32 && t.s3 % 32 == 0;
 }
 
 // ---------------------------------------------------------------- PAPER
+// Jacobi-1D, Section 4.1 as printed: Eqs. 3-9, Ttile by Eq. 10 (k = 1) or Eq. 12
+// (k > 1), Talg by Eq. 6.
+double talg_paper_1d(const int64_t* S, int64_t T, const stencil_tile& tl, const model_hw_params& hw) {
+    const int64_t tT = tl.t, tS = tl.s1, S1 = S[0];
+    const int64_t r = T - (T / tT) * tT;
+    const int64_t Nw = 2 * cdiv(T, tT) + ((r > 0 && 2 * r <= tT) ? 0 : 1);      // Eq. 3
+    const int64_t wtile = tS + tT - 2;                                          // Eq. 4
+    const int64_t w = cdiv(S1, 2 * tS + tT);                                    // Eq. 5
+    const double m_prime = 2.0 * (double)(tS + 2 * tT) * hw.L_s_per_word + 2.0 * hw.tau_sync_s;   // Eqs. 7-8
+    double sum = 0.0;
+    for (int64_t x = tS; x <= wtile; x += 2) sum += (double)cdiv(x, hw.n_v);
+    const double c = 2.0 * hw.C_iter_s * sum + (double)tT * hw.tau_sync_s;       // Eq. 9
+    const int64_t Mbytes = 4 * 2 * (tS + tT);                                    // Mtile = 2(wtile + 2)
+    if (Mbytes > hw.m_block_bytes) return std::numeric_limits<double>::infinity();
+    const int64_t k = std::min<int64_t>(hw.m_sm_bytes / Mbytes, hw.mtb_sm);     // Eq. 11 (reading M4)
+    if (k < 1) return std::numeric_limits<double>::infinity();
+    const double Ttile = k == 1 ? m_prime + c : m_prime + c + (double)(k - 1) * std::max(m_prime, c);   // Eq. 10/12
+    return (double)Nw * Ttile * (double)cdiv(cdiv(w, k), hw.n_sm) + (double)Nw * hw.T_sync_s;        // Eq. 6
+}
+
 double talg_paper(int nd, const int64_t* S, int64_t T, const stencil_tile& tl, const model_hw_params& hw) {
+    if (nd == 1) return talg_paper_1d(S, T, tl, hw);
     const int64_t tT = tl.t, tS1 = tl.s1, tS2 = tl.s2, tS3 = nd == 3 ? tl.s3 : 1;
     const int64_t S1 = S[0], S2 = S[1], S3 = nd == 3 ? S[2] : 1;
     // Eq. 3: Nw = 2 ceil(T/tT) + eps, eps = 0 iff 0 < T - floor(T/tT) tT <= tT/2
@@ -111,7 +134,7 @@ double talg_exact(int nd, const int64_t* S, int64_t T, const stencil_tile& tl, c
         // footprint (reads) and facets (writes) per unit inner extent, reading G3
         int64_t reads = 0, writes = 0, area = 0;
         double csum = 0.0;
-        const int64_t inner = nd == 2 ? tS2 : tS2 * tS3;
+        const int64_t inner = nd == 1 ? 1 : nd == 2 ? tS2 : tS2 * tS3;
         for (int64_t tau = lo; tau < hi; ++tau) {
             const int64_t W = row_width(tau, tS1, tT);
             area += W;
@@ -123,7 +146,11 @@ double talg_exact(int nd, const int64_t* S, int64_t T, const stencil_tile& tl, c
         }
         double Nsub, mi, mo, extra = 0.0;
         int64_t J = 1;
-        if (nd == 2) {
+        if (nd == 1) {
+            Nsub = 1.0;
+            mi = (double)reads;
+            mo = (double)writes;
+        } else if (nd == 2) {
             Nsub = (double)cdiv(S2 + nlev - 1, tS2);
             mi = (double)reads * (double)(tS2 + 2);
             mo = (double)writes * (double)tS2;
@@ -178,7 +205,7 @@ extern "C" double model_predict(stencil_kind kind, int ndims, const int64_t* dim
         if (dims[d] < 3) return nan;
     if (!tile_ok(ndims, tile)) return nan;
     if (hw->n_sm < 1 || hw->n_v < 1 || hw->mtb_sm < 1 || hw->m_sm_bytes < 1 || hw->m_block_bytes < 1) return nan;
-    int64_t S[3] = {dims[0] - 2, dims[1] - 2, ndims == 3 ? dims[2] - 2 : 1};
+    int64_t S[3] = {dims[0] - 2, ndims >= 2 ? dims[1] - 2 : 1, ndims == 3 ? dims[2] - 2 : 1};
     auto f = hw->geometry == 1 ? talg_exact : talg_paper;
     if (hw->n_gpus > 1) return talg_dist(ndims, S, T, tile, *hw, f);
     return f(ndims, S, T, tile, *hw);
@@ -191,7 +218,7 @@ extern "C" int model_select_tile(stencil_kind kind, int ndims, const int64_t* di
     for (int d = 0; d < ndims; ++d)
         if (dims[d] < 3) return STENCIL_EINVAL;
     // search space, reading M6
-    const int64_t S1 = dims[0] - 2, S2 = dims[1] - 2, S3 = ndims == 3 ? dims[2] - 2 : 1;
+    const int64_t S1 = dims[0] - 2, S2 = ndims >= 2 ? dims[1] - 2 : 1, S3 = ndims == 3 ? dims[2] - 2 : 1;
     const int64_t Tev = T + (T & 1);
     const int64_t tTmax = std::min<int64_t>(Tev, 128), tS1max = std::min<int64_t>(S1, 64);
     const int64_t innerS = ndims == 2 ? S2 : S3;
@@ -201,7 +228,19 @@ extern "C" int model_select_tile(stencil_kind kind, int ndims, const int64_t* di
     std::vector<V> vals;
     stencil_tile bt{0, 0, 0, 0};
     double bv = std::numeric_limits<double>::infinity();
-    for (int64_t tT = 2; tT <= tTmax; tT += 2)
+    if (ndims == 1) {
+        // reading M6 (1D): tS1 in 32..min(S1 rounded up to 32, 4096) step 32
+        const int64_t lim = std::min<int64_t>(cdiv(S1, 32) * 32, 4096);
+        for (int64_t tT = 2; tT <= tTmax; tT += 2)
+            for (int64_t tS1 = 32; tS1 <= lim; tS1 += 32) {
+                const stencil_tile t{(int)tT, (int)tS1, 0, 0};
+                const double v = model_predict(kind, ndims, dims, T, t, hw);
+                if (!std::isfinite(v)) continue;
+                vals.push_back(V{t, v});
+                if (v < bv) { bv = v; bt = t; }
+            }
+    }
+    for (int64_t tT = 2; ndims > 1 && tT <= tTmax; tT += 2)
         for (int64_t tS1 = 1; tS1 <= tS1max; ++tS1) {
             const int64_t n2 = ndims == 2 ? 1 : tS2max3;
             for (int64_t a = 1; a <= n2; ++a)

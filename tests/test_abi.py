@@ -175,3 +175,42 @@ def test_exact_fit_recovers_constants(lib):
     fit = tune.fit_exact(hhc.HEAT2D_9PT, insts)
     assert abs(fit["C_iter_s"] / C - 1) < 1e-6 and abs(fit["tau_level_s"] / tau - 1) < 1e-6
     assert fit["rel_rmse"] < 1e-9
+
+
+# ---- Jacobi-1D: the paper's 1D model (Section 4.1) and the library agree
+@pytest.mark.parametrize("geometry", [hhc.PAPER, hhc.EXACT])
+def test_model_1d_matches_oracle(lib, geometry):
+    rnd = random.Random(geometry + 70)
+    n = 0
+    for _ in range(200):
+        o, c = hw_pair(1, geometry, rnd, b200=rnd.random() < 0.5)   # C_iter: a parameter (Table 4 has no 1D row)
+        S = (rnd.randint(1, 10 ** 6),)
+        tile = (2 * rnd.randint(1, 200), rnd.randint(1, 3000), 0, 0)
+        T = rnd.randint(1, 2000)
+        got = hhc.model_predict(hhc.JACOBI1D_3PT, (S[0] + 2,), T, tile, c)
+        exp = mo.talg(1, S, T, tile, o)
+        if math.isinf(exp):
+            assert math.isinf(got)
+        else:
+            n += 1
+            assert abs(got - exp) <= 1e-12 * exp, (S, T, tile, got, exp)
+    assert n > 100
+    o, c = hw_pair(1, geometry, b200=True)
+    best, thr, cands = hhc.model_select_tile(hhc.JACOBI1D_3PT, (3000,), 40, c, 0.10)
+    ob, ot, oc = mo.select_tile(1, (2998,), 40, o, 0.10)
+    assert best == ob and cands == oc and thr == 256
+
+
+def test_model_1d_hand_example():
+    """Eqs. 3-9, 10 and 6 by hand for S = 1000, T = 10, tile (4, 8), GTX 980 constants (Jacobi2D C_iter):
+    Nw = 2*ceil(10/4) + eps = 6 (r = 10 - 8 = 2 <= tT/2 -> eps = 0); w = ceil(1000/20) = 50;
+    mio = 2(8+8) = 32 words; wtile = 10: c = 2 Citer (ceil(8/128) + ceil(10/128)) + 4 tau = 4 Citer + 4 tau;
+    Mtile = 2(8+4) = 24 words = 96 B -> k = min(98304 // 96, 32) = 32 -> Ttile = m' + c + 31 max(m', c);
+    rounds = ceil(ceil(50/32)/16) = 1."""
+    o = mo.gtx980(1, mo.PAPER)
+    Nw, w = 6, 50
+    m = 32 * o.L + 2 * o.tau_sync
+    c = 4 * o.C_iter + 4 * o.tau_sync
+    Ttile = m + c + 31 * max(m, c)
+    exp = Nw * Ttile * 1 + Nw * o.T_sync
+    assert abs(mo.talg(1, (1000,), 10, (4, 8, 0, 0), o) - exp) <= 1e-15 * exp

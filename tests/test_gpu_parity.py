@@ -289,3 +289,29 @@ def test_parity_pair_layout(kind, mode):
         coeffs = [float(x) * 0.95 for x in w] + [0.003]
         exp = oracle.run(kind, a, 11, mode, coeffs=coeffs)
         assert_bits(gpu_run(kind, a, 11, (4, 3, 512), mode, coeffs=coeffs), exp, "pair coeffs")
+
+
+# ---- Jacobi-1D: K0, one block per hexagon
+@pytest.mark.parametrize("mode", [hhc.PLAIN, hhc.FUSED])
+def test_parity_1d(mode):
+    rng = np.random.default_rng(70 + mode)
+    for tile in [(2, 1), (4, 3), (8, 32), (16, 100), (64, 512), (6, 2000)]:
+        n = int(rng.integers(3, 5000))
+        a = field(int(rng.integers(1, 1 << 30)), (n,))
+        for T in (1, 2, 7, tile[0] + 1, 3 * tile[0] + 5):
+            exp = oracle.run(hhc.JACOBI1D_3PT, a, T, mode)
+            got = gpu_run(hhc.JACOBI1D_3PT, a, T, tile, mode)
+            assert_bits(got, exp, f"1D n {n} T {T} tile {tile}")
+
+
+def test_parity_1d_large_and_coeffs():
+    a = field(71, (1_000_003,))
+    for T, tile in ((100, (32, 2048)), (257, (64, 4096))):
+        assert_bits(gpu_run(hhc.JACOBI1D_3PT, a, T, tile), oracle.run(hhc.JACOBI1D_3PT, a, T, hhc.FUSED),
+                    f"1D large T {T}")
+    coeffs = [0.25, 0.5, 0.25, 0.001]
+    for mode in (hhc.PLAIN, hhc.FUSED):
+        assert_bits(gpu_run(hhc.JACOBI1D_3PT, a[:20001], 33, (8, 256), mode, coeffs=coeffs),
+                    oracle.run(hhc.JACOBI1D_3PT, a[:20001], 33, mode, coeffs=coeffs), "1D coeffs")
+    plain = oracle.run(hhc.JACOBI1D_3PT, a, 100, hhc.PLAIN)
+    assert max_rel(gpu_run(hhc.JACOBI1D_3PT, a, 100, (32, 2048), hhc.FUSED), plain) <= 1e-5

@@ -311,3 +311,57 @@ def test_rejects_bad_arguments():
         oracle.run(HEAT2D_9PT, a, -1)
     with pytest.raises(ValueError):
         oracle.run(HEAT2D_9PT, a, 1, coeffs=[1.0, 2.0])
+
+
+# ------------------------------------------------------------------ Jacobi-1D
+# The 1D 3-point average the paper's derivation starts from (Eqs. 2-12);
+# weights fp32(1/3) each (reading R1, PolyBench jacobi-1d), canonical order.
+
+def test_jacobi1d_hand_values():
+    # (3 + 6 + 9)/3: w*3 = 1.00000003 -> 1, w*6 -> 2 (+ 1 = 3), w*9 -> 3 (+ 3 = 6) in both modes
+    g = np.array([3.0, 6.0, 9.0], np.float32)
+    for mode in (PLAIN, FUSED):
+        out = oracle.run(oracle.JACOBI1D_3PT, g, 1, mode)
+        assert out[1] == F32(6.0) and out[0] == g[0] and out[2] == g[2], (mode, out)
+    offs, w = oracle.stencil_info(oracle.JACOBI1D_3PT)
+    assert [tuple(o) for o in offs] == [(-1, 0, 0), (0, 0, 0), (1, 0, 0)]
+    assert all(x == F32(1.0) / F32(3.0) for x in w)
+
+
+@pytest.mark.parametrize("mode", [PLAIN, FUSED])
+def test_jacobi1d_brute_force_bit_exact(mode):
+    a = field(107, (12,))
+    for T in (0, 1, 2, 5, 9):
+        got = oracle.run(oracle.JACOBI1D_3PT, a, T, mode)
+        exp = brute_force(oracle.JACOBI1D_3PT, a, T, mode)
+        assert np.array_equal(got.view(np.uint32), exp.view(np.uint32)), (mode, T)
+
+
+def test_jacobi1d_dense_matrix_and_fourier():
+    kind = oracle.JACOBI1D_3PT
+    a = field(9, (40,))
+    M = iteration_matrix(kind, (40,))
+    x = a.astype(np.float64)
+    for _ in range(30):
+        x = M @ x
+    for mode in (PLAIN, FUSED):
+        got = oracle.run(kind, a, 30, mode).astype(np.float64)
+        assert np.max(np.abs(got - x)) <= 4 * 30 * 3 * 2.0 ** -24
+    # sine mode with a zero ring: u_T = lambda^T u_0, lambda = w (1 + 2 cos theta)
+    n, p, T = 101, 7, 50
+    th = np.pi * p / (n - 1)
+    u = np.sin(th * np.arange(n))
+    u[0] = u[-1] = 0.0
+    w = float(F32(1.0) / F32(3.0))
+    lam = w * (1 + 2 * np.cos(th))
+    for mode in (PLAIN, FUSED):
+        got = oracle.run(kind, u.astype(np.float32), T, mode).astype(np.float64)
+        assert np.max(np.abs(got - lam ** T * u)) <= (4 * T * 3 + 2) * 2.0 ** -24
+
+
+def test_jacobi1d_fused_vs_plain_and_threads():
+    a = field(5, (5001,))
+    p = oracle.run(oracle.JACOBI1D_3PT, a, 64, PLAIN)
+    f = oracle.run(oracle.JACOBI1D_3PT, a, 64, FUSED)
+    assert np.max(np.abs(f.astype(np.float64) - p) / np.maximum(np.abs(p), 2.0 ** -10)) <= 1e-5
+    assert np.array_equal(oracle.run(oracle.JACOBI1D_3PT, a, 64, FUSED, nthreads=1), f)
