@@ -40,7 +40,7 @@ CONFIGS = {
     "C5": dict(kind=5, dims=(768, 768, 768), T=128, tile=(8, 6, 8, 64), threads=256,
                desc="Laplacian-3D 27-point fp32, 768^3, T=128"),
     # SURVEY §8(f) f2 (not a BASELINE.json config): the paper's 1D derivation case
-    "X1": dict(kind=7, dims=(1 << 26,), T=1024, tile=(64, 2048), threads=256,
+    "X1": dict(kind=7, dims=(1 << 26,), T=1024, tile=(128, 2048), threads=256,
                desc="Jacobi-1D 3-point fp32, 2^26 points, T=1024 (extension f2)"),
 }
 DEFAULT_CONFIG = "C2"
