@@ -36,7 +36,8 @@ KINDS = [hhc.JACOBI2D_5PT, hhc.HEAT2D_9PT, hhc.LAPLACIAN2D_5PT, hhc.GRADIENT2D, 
          hhc.LAPLACIAN3D_27PT]
 
 
-def b200_hw(cal: dict | None, kind: int, geometry: int, threads: int = 0) -> "hhc.model_hw_params":
+def b200_hw(cal: dict | None, kind: int, geometry: int, threads: int = 0,
+            leff: bool = False) -> "hhc.model_hw_params":
     """Table 2 analogue for B200 plus calibrated Table 3/4 constants."""
     import torch
     props = torch.cuda.get_device_properties(0) if torch.cuda.is_available() else None
@@ -52,7 +53,46 @@ def b200_hw(cal: dict | None, kind: int, geometry: int, threads: int = 0) -> "hh
         if geometry == hhc.EXACT and fit:
             hw.C_iter_s = fit["C_iter_s"]
             hw.tau_sync_s = fit["tau_level_s"]
+        lf = (cal.get("exact_leff") or {}).get(str(kind))
+        if leff and geometry == hhc.EXACT and lf:
+            hw.L_s_per_word = lf["L_s_per_word"]
     return hw
+
+
+def fit_leff(cal: dict, kind: int, full):
+    """Reading Q14b (EXACT-Leff, not the paper's procedure): with C_iter / tau
+    from the compute-only fit, the per-word data-movement cost L is fitted to
+    FULL runs of the calibration instances (relative least squares, golden
+    section on log L) instead of taken from the copy micro-benchmark: it then
+    carries what moving a footprint word costs the implemented kernels (LSU
+    issue of the 4-16 B cp.async, the S2-face hand-off), which the copy
+    bandwidth does not."""
+    def err(logL):
+        e, n = 0.0, 0
+        for dims, T, tile, t in full:
+            hw = b200_hw(cal, kind, hhc.EXACT)
+            hw.L_s_per_word = math.exp(logL)
+            v = hhc.model_predict(kind, dims, T, tile, hw)
+            if math.isfinite(v) and t > 0:
+                e += ((v - t) / t) ** 2
+                n += 1
+        return math.sqrt(e / max(n, 1)), n
+    lo, hi = math.log(cal["L_s_per_word"] / 10), math.log(cal["L_s_per_word"] * 1000)
+    g = (math.sqrt(5) - 1) / 2
+    a, b = hi - g * (hi - lo), lo + g * (hi - lo)
+    fa, fb = err(a)[0], err(b)[0]
+    for _ in range(40):
+        if fa < fb:
+            hi, b, fb = b, a, fa
+            a = hi - g * (hi - lo)
+            fa = err(a)[0]
+        else:
+            lo, a, fa = a, b, fb
+            b = lo + g * (hi - lo)
+            fb = err(b)[0]
+    x = (lo + hi) / 2
+    e, n = err(x)
+    return {"L_s_per_word": math.exp(x), "rel_rmse": e, "n": n}
 
 
 def load_cal(path=None):
@@ -93,7 +133,7 @@ def calibrate(args):
     out["tau_sync_s"] = hhc.stencil_microbench(1, threads=256)
     out["T_sync_s"] = hhc.stencil_microbench(2)
     rnd = random.Random(2017)
-    citer, samples, fits, insts, raw = {}, {}, {}, [], {}
+    citer, samples, fits, insts, raw, full, full_all = {}, {}, {}, [], {}, [], {}
     for kind in KINDS:
         nd = hhc.KIND_NDIMS[kind]
         vals = []
@@ -113,21 +153,31 @@ def calibrate(args):
             if math.isfinite(v) and v > 0:
                 vals.append(v)
                 insts.append((dims, T, tile, v))
+                # the same instance run for real (for reading Q14b's L fit)
+                h = hhc.stencil_create(kind, dims)
+                a = torch.rand(*dims, device="cuda")
+                b = torch.empty_like(a)
+                full.append((dims, T, tile, time_run(h, a, b, T, tile, 0, reps=2)))
+                hhc.stencil_destroy(h)
         citer[str(kind)] = sum(vals) / len(vals)
         samples[str(kind)] = {"n": len(vals), "min": min(vals), "max": max(vals)}
         fits[str(kind)] = fit_exact(kind, insts)
+        full_all[str(kind)] = list(full)
         raw[str(kind)] = [[list(d), T_, list(t), v] for d, T_, t, v in insts]
         insts.clear()
+        full.clear()
         print(f"C_iter kind {kind}: {citer[str(kind)]:.3e} s over {len(vals)} instances; "
               f"EXACT fit {fits[str(kind)]}", flush=True)
     out["C_iter_s"] = citer
     out["C_iter_samples"] = samples
     out["exact_fit"] = fits
     out["instances"] = raw          # (dims, T, tile, compute-only seconds): refits need no GPU
+    out["exact_leff"] = {k: fit_leff(out, int(k), v) for k, v in full_all.items()}
+    out["instances_full"] = {k: [[list(d), T_, list(t), v] for d, T_, t, v in f] for k, f in full_all.items()}
     os.makedirs(os.path.dirname(args.out), exist_ok=True)
     with open(args.out, "w") as f:
         json.dump(out, f, indent=1)
-    print(json.dumps({k: v for k, v in out.items() if k not in ("C_iter_samples", "instances")}))
+    print(json.dumps({k: v for k, v in out.items() if k not in ("C_iter_samples", "instances", "instances_full")}))
 
 
 def _basis(kind, dims, T, tile, c_iter, tau):
@@ -224,16 +274,23 @@ def sweep(args):
         p = {"tile": list(tile), "threads": threads, "texec": te}
         for geom, name in ((hhc.PAPER, "talg_paper"), (hhc.EXACT, "talg_exact")):
             p[name] = hhc.model_predict(kind, dims, T, tile, b200_hw(cal, kind, geom, threads))
+        if (cal.get("exact_leff") or {}).get(str(kind)):
+            p["talg_exact_leff"] = hhc.model_predict(kind, dims, T, tile,
+                                                     b200_hw(cal, kind, hhc.EXACT, threads, leff=True))
         pts.append(p)
         print(json.dumps(p), flush=True)
     best = min(pts, key=lambda p: p["texec"])
     res = {"config": args.config, "n_points": len(pts), "best_measured": best, "points": pts}
-    for name in ("talg_paper", "talg_exact"):
+    for name in ("talg_paper", "talg_exact", "talg_exact_leff"):
+        if not all(name in p for p in pts):
+            continue
         ra, rn, nn = stats(pts, name)
         res[name] = {"rmse_all": ra, "rmse_within_20pct": rn, "n_within_20pct": nn}
     # chosen-tile gaps (reading Q17), model argmin over the swept points and over Eq. 31's space
-    for geom, name in ((hhc.PAPER, "paper"), (hhc.EXACT, "exact")):
-        hw = b200_hw(cal, kind, geom)
+    for geom, name, lf in ((hhc.PAPER, "paper", False), (hhc.EXACT, "exact", False), (hhc.EXACT, "exact_leff", True)):
+        if lf and not (cal.get("exact_leff") or {}).get(str(kind)):
+            continue
+        hw = b200_hw(cal, kind, geom, leff=lf)
         try:
             bt, bthr, cands = hhc.model_select_tile(kind, dims, T, hw, 0.10)
             te = time_run(h, d_in, d_out, T, bt, bthr, reps=args.reps)

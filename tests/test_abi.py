@@ -214,3 +214,25 @@ def test_model_1d_hand_example():
     Ttile = m + c + 31 * max(m, c)
     exp = Nw * Ttile * 1 + Nw * o.T_sync
     assert abs(mo.talg(1, (1000,), 10, (4, 8, 0, 0), o) - exp) <= 1e-15 * exp
+
+
+def test_leff_fit_recovers_L(lib):
+    """tune.fit_leff (reading Q14b): full-run times generated by the EXACT model
+    with a known per-word cost L* are fitted back to L* (C_iter/tau held)."""
+    from paper_conf_ppopp_prajapatirradg17_b200 import tune
+    cal = {"L_s_per_word": 6.5e-13, "tau_sync_s": 1.5e-8, "T_sync_s": 5.4e-7, "C_iter_s": {"4": 4e-9},
+           "exact_fit": {"4": {"C_iter_s": 4e-9, "tau_level_s": 5e-10}}}
+    rnd = random.Random(3)
+    Lstar = 2.1e-11
+    full = []
+    for _ in range(25):
+        dims = (rnd.randint(96, 256), rnd.randint(96, 256), rnd.randint(96, 256))
+        tile = (2 * rnd.randint(1, 6), rnd.randint(1, 8), rnd.randint(1, 6), 32 * rnd.randint(1, 2))
+        T = rnd.randint(8, 24)
+        hw = tune.b200_hw(cal, 4, hhc.EXACT)
+        hw.L_s_per_word = Lstar
+        t = hhc.model_predict(4, dims, T, tile, hw)
+        if math.isfinite(t):
+            full.append((dims, T, tile, t))
+    fit = tune.fit_leff(cal, 4, full)
+    assert abs(fit["L_s_per_word"] / Lstar - 1) < 1e-3 and fit["rel_rmse"] < 1e-3 and fit["n"] == len(full)
