@@ -107,7 +107,7 @@ int run_microbench(int which, int kind, int ndims, const int64_t* dims, int64_t 
         stencil_t h = nullptr;
         rc = stencil_create((stencil_kind)kind, ndims, dims, nullptr, 0, STENCIL_MODE_FUSED, &h);
         if (rc == STENCIL_OK) {
-            const int64_t n = dims[0] * dims[1] * (ndims == 3 ? dims[2] : 1);
+            const int64_t n = dims[0] * (ndims >= 2 ? dims[1] : 1) * (ndims == 3 ? dims[2] : 1);
             float *a = nullptr, *b = nullptr;
             if (cudaMalloc(&a, n * 4) != cudaSuccess || cudaMalloc(&b, n * 4) != cudaSuccess) rc = STENCIL_ENOMEM;
             if (rc == STENCIL_OK) {

@@ -33,7 +33,7 @@ if ROOT not in sys.path:
 import paper_conf_ppopp_prajapatirradg17_b200 as hhc  # noqa: E402
 
 KINDS = [hhc.JACOBI2D_5PT, hhc.HEAT2D_9PT, hhc.LAPLACIAN2D_5PT, hhc.GRADIENT2D, hhc.HEAT3D_7PT,
-         hhc.LAPLACIAN3D_27PT]
+         hhc.LAPLACIAN3D_27PT, hhc.JACOBI1D_3PT]
 
 
 def b200_hw(cal: dict | None, kind: int, geometry: int, threads: int = 0,
@@ -119,6 +119,8 @@ def time_run(h, d_in, d_out, T, tile, threads, reps=3):
 
 
 def random_tile(rnd, nd, dims):
+    if nd == 1:
+        return (2 * rnd.randint(1, 64), 32 * rnd.randint(1, 128), 0, 0)
     if nd == 2:
         return (2 * rnd.randint(1, 16), rnd.randint(1, 32), 32 * rnd.randint(1, 16), 0)
     return (2 * rnd.randint(1, 6), rnd.randint(1, 8), rnd.randint(1, 6), 32 * rnd.randint(1, 2))
@@ -128,17 +130,28 @@ def calibrate(args):
     out = {"device": None, "how": "PAPER.md §5.2 micro-benchmarks re-measured on this GPU"}
     import torch
     out["device"] = torch.cuda.get_device_name(0)
-    out["L_s_per_word"] = hhc.stencil_microbench(0)
-    out["L_s_per_GB"] = out["L_s_per_word"] / 4e-9
-    out["tau_sync_s"] = hhc.stencil_microbench(1, threads=256)
-    out["T_sync_s"] = hhc.stencil_microbench(2)
+    kinds = [int(k) for k in args.kinds.split(",")] if getattr(args, "kinds", None) else KINDS
+    base = None
+    if getattr(args, "base", None):
+        # add kinds to an existing calibration (its L, tau_sync, T_sync and other kinds kept)
+        base = load_cal(args.base)
+        for k in ("L_s_per_word", "L_s_per_GB", "tau_sync_s", "T_sync_s"):
+            out[k] = base[k]
+    else:
+        out["L_s_per_word"] = hhc.stencil_microbench(0)
+        out["L_s_per_GB"] = out["L_s_per_word"] / 4e-9
+        out["tau_sync_s"] = hhc.stencil_microbench(1, threads=256)
+        out["T_sync_s"] = hhc.stencil_microbench(2)
     rnd = random.Random(2017)
     citer, samples, fits, insts, raw, full, full_all = {}, {}, {}, [], {}, [], {}
-    for kind in KINDS:
+    for kind in kinds:
         nd = hhc.KIND_NDIMS[kind]
         vals = []
         while len(vals) < args.instances:
-            if nd == 2:
+            if nd == 1:
+                dims = (rnd.randint(100000, 2000000),)
+                T = rnd.randint(16, 64)
+            elif nd == 2:
                 dims = (rnd.randint(1024, 4096), rnd.randint(1024, 4096))
                 T = rnd.randint(16, 64)
             else:
@@ -168,12 +181,21 @@ def calibrate(args):
         full.clear()
         print(f"C_iter kind {kind}: {citer[str(kind)]:.3e} s over {len(vals)} instances; "
               f"EXACT fit {fits[str(kind)]}", flush=True)
-    out["C_iter_s"] = citer
-    out["C_iter_samples"] = samples
-    out["exact_fit"] = fits
-    out["instances"] = raw          # (dims, T, tile, compute-only seconds): refits need no GPU
-    out["exact_leff"] = {k: fit_leff(out, int(k), v) for k, v in full_all.items()}
-    out["instances_full"] = {k: [[list(d), T_, list(t), v] for d, T_, t, v in f] for k, f in full_all.items()}
+    if base is not None:
+        for key, new in (("C_iter_s", citer), ("C_iter_samples", samples), ("exact_fit", fits), ("instances", raw)):
+            merged = dict(base.get(key) or {})
+            merged.update(new)
+            out[key] = merged
+        out["exact_leff"] = dict(base.get("exact_leff") or {})
+        out["instances_full"] = dict(base.get("instances_full") or {})
+    else:
+        out["C_iter_s"] = citer
+        out["C_iter_samples"] = samples
+        out["exact_fit"] = fits
+        out["instances"] = raw          # (dims, T, tile, compute-only seconds): refits need no GPU
+        out["exact_leff"], out["instances_full"] = {}, {}
+    out["exact_leff"].update({k: fit_leff(out, int(k), v) for k, v in full_all.items()})
+    out["instances_full"].update({k: [[list(d), T_, list(t), v] for d, T_, t, v in f] for k, f in full_all.items()})
     os.makedirs(os.path.dirname(args.out), exist_ok=True)
     with open(args.out, "w") as f:
         json.dump(out, f, indent=1)
@@ -219,6 +241,9 @@ def fit_exact(kind, insts):
 def sweep_tiles(nd, limit):
     """A bounded grid of feasible tiles (x threads choices): the B200 analogue of
     the paper's baseline experiments (85 tiles x 10 thread counts)."""
+    if nd == 1:
+        return [((tT, tS1, 0, 0), 256) for tT in (4, 8, 16, 32, 64, 128, 256)
+                for tS1 in (128, 256, 512, 1024, 2048, 4096)][:limit]
     if nd == 2:
         tiles = [(tT, tS1, tS2, 0) for tT in (4, 8, 12, 16, 24, 32) for tS1 in (4, 8, 12, 16, 20, 28)
                  for tS2 in (128, 256, 512)]
@@ -345,6 +370,8 @@ def main(argv=None):
     c = sub.add_parser("calibrate")
     c.add_argument("--out", default=os.path.join(ROOT, "profiles", "hw_params_b200.json"))
     c.add_argument("--instances", type=int, default=70)
+    c.add_argument("--kinds", default=None, help="comma-separated kinds (default: all)")
+    c.add_argument("--base", default=None, help="existing calibration to extend (its global constants kept)")
     s = sub.add_parser("sweep")
     s.add_argument("--config", default="C2")
     s.add_argument("--cal", default=None)
