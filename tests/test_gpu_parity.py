@@ -315,3 +315,85 @@ def test_parity_1d_large_and_coeffs():
                     oracle.run(hhc.JACOBI1D_3PT, a[:20001], 33, mode, coeffs=coeffs), "1D coeffs")
     plain = oracle.run(hhc.JACOBI1D_3PT, a, 100, hhc.PLAIN)
     assert max_rel(gpu_run(hhc.JACOBI1D_3PT, a, 100, (32, 2048), hhc.FUSED), plain) <= 1e-5
+
+
+# ---- the overlapped multi-GPU loop (dist.run_slabs_overlap) on ONE GPU: virtual ranks in threads, each
+# with its own streams and handles, a queue-backed stand-in for torch.distributed's P2P (device copies
+# ordered by CUDA events).  Exercises the stream/event logic of the GPU path, not NCCL itself.
+class _Work:
+    def __init__(self, q, buf):
+        self.q, self.buf = q, buf
+
+    def wait(self):
+        t, ev = self.q.get(timeout=120)
+        torch.cuda.current_stream().wait_event(ev)
+        self.buf.copy_(t)
+
+
+class _FakeDist:
+    isend, irecv = "isend", "irecv"
+
+    class P2POp:
+        def __init__(self, op, tensor, peer):
+            self.op, self.tensor, self.peer = op, tensor, peer
+
+    def __init__(self, rank, board):
+        self.rank, self.board = rank, board
+
+    def batch_isend_irecv(self, ops):
+        works = []
+        for o in ops:
+            if o.op == "isend":
+                t = o.tensor.clone()
+                ev = torch.cuda.Event()
+                ev.record()
+                self.board[(self.rank, o.peer)].put((t, ev))
+            else:
+                works.append(_Work(self.board[(o.peer, self.rank)], o.tensor))
+        return works
+
+
+@pytest.mark.parametrize("kind,dims,T,tT,world", [
+    (hhc.HEAT2D_9PT, (2 * 160 + 2, 300), 37, 8, 2),
+    (hhc.GRADIENT2D, (3 * 60 + 2, 130), 21, 4, 3),
+    (hhc.HEAT3D_7PT, (2 * 40 + 2, 30, 70), 13, 4, 2),
+])
+def test_overlapped_slabs_gpu_streams(kind, dims, T, tT, world):
+    import queue
+    import threading
+    from paper_conf_ppopp_prajapatirradg17_b200 import dist as hdist
+    a = field(98, dims)
+    tile = (tT, 3, 32) if len(dims) == 2 else (tT, 2, 3, 32)
+    board = {(i, j): queue.Queue() for i in range(world) for j in range(world)}
+    out, errs = {}, []
+
+    def rank_main(r):
+        try:
+            torch.cuda.set_device(0)
+            s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+            with torch.cuda.stream(s1):
+                slab = hdist.partition(dims[0], world, r, tT)
+                ext = (slab.rows,) + dims[1:]
+                h, he = hhc.stencil_create(kind, ext), hhc.stencil_create(kind, ext)
+                p0 = torch.from_numpy(np.ascontiguousarray(a[slab.e0:slab.e1])).to(DEV)
+                p1 = torch.empty_like(p0)
+                res = hdist.run_slabs_overlap(slab, p0, p1, T, tT, hdist.gpu_stepper(h, tile, 0, s1),
+                                              hdist.gpu_stepper(he, tile, 0, s2), _FakeDist(r, board), (s1, s2))
+                lo, hi = slab.held
+                out[r] = (lo, hi, res[lo - slab.e0:hi - slab.e0].cpu().numpy())
+                torch.cuda.synchronize()
+                hhc.stencil_destroy(h)
+                hhc.stencil_destroy(he)
+        except Exception as e:          # surfaced below
+            errs.append(e)
+
+    ts = [threading.Thread(target=rank_main, args=(r,)) for r in range(world)]
+    for t in ts:
+        t.start()
+    for t in ts:
+        t.join(300)
+    assert not errs, errs
+    exp = oracle.run(kind, a, T, hhc.FUSED)
+    for r in range(world):
+        lo, hi, got = out[r]
+        assert_bits(np.ascontiguousarray(got), np.ascontiguousarray(exp[lo:hi]), f"rank {r}")
