@@ -6,7 +6,7 @@
  * Stencils" (PPoPP'17).  Citations "P:Lnnn" are PAPER.md lines.
  *
  *   stencil_create / stencil_run  -- iterative stencil of Eq. 1
- *       time-stepped T times under hybrid hexagonal/classic (HHC) tiling
+ *       (1D, 2D or 3D) time-stepped T times under hybrid hexagonal/classic (HHC) tiling
  *       (§3.1; Fig. 1-2): hexagons of base tS1 and height tT over
  *       (t, S1), classic time skewing over S2 (and S3), one kernel launch per
  *       row of hexagons, one thread block per hexagonal prism/slab
@@ -65,7 +65,8 @@ typedef enum { STENCIL_MODE_PLAIN = 0, STENCIL_MODE_FUSED = 1 } stencil_mode;
 /* Tile sizes: the decision variables of Eq. 31.
  *   t  = tT  (even, >= 2), s1 = tS1 (>= 1), hexagon base along S1;
  *   2D: s2 = tS2, a multiple of 32 (inner, contiguous); s3 = 0.
- *   3D: s2 = tS2 >= 1 (middle), s3 = tS3, a multiple of 32 (inner). */
+ *   3D: s2 = tS2 >= 1 (middle), s3 = tS3, a multiple of 32 (inner).
+ *   1D (Jacobi-1D): s2 = s3 = 0; 256 threads per hexagon. */
 typedef struct { int32_t t, s1, s2, s3; } stencil_tile;
 
 /* Table 1 hardware parameters (EH) + C_iter (CSH); Table 2-4. */
