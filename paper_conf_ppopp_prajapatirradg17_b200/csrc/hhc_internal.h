@@ -39,7 +39,7 @@ struct HexParams {
 inline int64_t smem_bytes(int ndims, int tT, int tS1, int tS2, int tS3) {
     const int64_t NX = tS1 + tT + 2;
     const int64_t geo = 16 * (int64_t)tT;              // per-level geometry table (ints)
-    if (ndims == 1) return 4 * (((2 * NX + 3) & ~3) + geo);   // K0: two planes of NX values (16-B padded) + geometry
+    if (ndims == 1) return 4 * (2 * ((NX + 3) & ~3) + geo);   // K0: two 16-B padded planes of NX values + geometry
     if (ndims == 2) return 4 * ((2 * NX + 1) * (tS2 + 8) + 2 * (int64_t)tT * NX * 2 + geo + NX + 2 * (int64_t)tT + 2 + 2 * NX);
     return 4 * (2 * NX * (tS2 + 2) * (tS3 + 4) + 2 * (int64_t)tT * NX * (tS2 + 2) * 2 + geo);
 }
