@@ -176,6 +176,36 @@ int stencil_run_planes(stencil_t h, int64_t rows, float* plane0, float* plane1, 
 int stencil_profile(stencil_t h, const float* d_in, float* d_out, int64_t T, stencil_tile tile,
                     int threads, void* cuda_stream, double* kernel_seconds, int64_t* kernel_launches);
 
+/* ---- Wavefront-parallel Jacobi-1D (reading W1).
+ * The paper's generality claim, P:L1160-1170 ("Consider, wavefront parallel
+ * Jacobi1D stencil. The total execution time is the sum of the times for each
+ * wavefront ... equation 6 holds for wavefront parallel codes"): a second
+ * schedule of the same Eq. 1 update.  Parallelogram tiles of tile.t levels x
+ * tile.s1 columns in skewed coordinates x' = x + t; tile (i, j) covers the
+ * levels (i*t, min((i+1)*t, T)] and x' in [j*s1, (j+1)*s1); one kernel launch
+ * per anti-diagonal i + j (the wavefront), one thread block per tile.
+ * tile.t in [1, 1024] (any parity), tile.s1 in [2, 16384]; s2, s3 ignored. */
+
+/* A_T from A_0 like stencil_run (same pointer rules, stream-ordered,
+ * asynchronous, scratch plane owned by the handle), on a handle created for
+ * STENCIL_JACOBI1D_3PT (else STENCIL_EINVAL).  Not graph-captured: one launch
+ * per wavefront plus two set-up copies. */
+int stencil_run_wavefront(stencil_t h, const float* d_in, float* d_out, int64_t T,
+                          stencil_tile tile, void* cuda_stream);
+
+/* Schedule of a wavefront run on dims[0] points: number of wavefronts
+ * (launches), tiles in total and in the widest wavefront (host only). */
+int stencil_wavefront_info(const int64_t* dims, int64_t T, stencil_tile tile,
+                           int64_t* n_wavefronts, int64_t* n_tiles, int64_t* max_width);
+
+/* Talg of the wavefront schedule in seconds: Eq. 6 summed per wavefront, each
+ * with its own tile count, Ttile by Eqs. 8-12 on the parallelogram's
+ * footprint (reading W1).  hw->geometry selects L per word (PAPER)
+ * or per SM (EXACT, reading M5).  NaN for invalid arguments, +INFINITY for a
+ * tile that does not fit m_block_bytes. */
+double model_predict_wavefront(stencil_kind kind, int ndims, const int64_t* dims, int64_t T,
+                               stencil_tile tile, const model_hw_params* hw);
+
 /* Human-readable status. */
 const char* stencil_strerror(int status);
 

@@ -115,6 +115,11 @@ def load(build_if_missing: bool = False):
                                     P(ctypes.c_double), P(ctypes.c_int64)]
     lib.stencil_last_launches.argtypes = [vp]
     lib.stencil_last_launches.restype = ctypes.c_int64
+    lib.stencil_run_wavefront.argtypes = [vp, vp, vp, ctypes.c_int64, stencil_tile, vp]
+    lib.stencil_wavefront_info.argtypes = [i64p, ctypes.c_int64, stencil_tile, i64p, i64p, i64p]
+    lib.model_predict_wavefront.argtypes = [ctypes.c_int, ctypes.c_int, i64p, ctypes.c_int64, stencil_tile,
+                                            P(model_hw_params)]
+    lib.model_predict_wavefront.restype = ctypes.c_double
     _lib = lib
     return lib
 
@@ -216,6 +221,26 @@ def stencil_profile(s: Stencil, d_in, d_out, T: int, tile, threads: int = 0, str
     return sec.value, n.value
 
 
+def stencil_run_wavefront(s: Stencil, d_in, d_out, T: int, tile, stream=None):
+    """Wavefront-parallel Jacobi-1D (hhc.h): tile = (t, s1) parallelogram."""
+    _check(load().stencil_run_wavefront(s.handle, _ptr(d_in), _ptr(d_out), int(T), make_tile(tile),
+                                        _stream(stream)), "stencil_run_wavefront")
+
+
+def stencil_wavefront_info(dims, T: int, tile):
+    """(wavefronts = launches, tiles in total, tiles of the widest wavefront)."""
+    d, _ = _dims(dims)
+    out = [ctypes.c_int64() for _ in range(3)]
+    _check(load().stencil_wavefront_info(d, int(T), make_tile(tile), *[ctypes.byref(o) for o in out]),
+           "stencil_wavefront_info")
+    return tuple(o.value for o in out)
+
+
+def model_predict_wavefront(dims, T: int, tile, hw: model_hw_params) -> float:
+    d, nd = _dims(dims)
+    return float(load().model_predict_wavefront(JACOBI1D_3PT, nd, d, int(T), make_tile(tile), ctypes.byref(hw)))
+
+
 def stencil_last_launches(s: Stencil) -> int:
     return int(load().stencil_last_launches(s.handle))
 
@@ -272,4 +297,5 @@ def updates(dims, T: int) -> int:
 EXPORTED_SYMBOLS = ["stencil_create", "stencil_destroy", "stencil_run", "stencil_run_host",
                     "stencil_run_planes", "model_predict", "model_select_tile", "stencil_tile_resources",
                     "stencil_plan_info", "stencil_microbench", "stencil_strerror", "stencil_last_launches",
-                    "stencil_profile"]
+                    "stencil_profile", "stencil_run_wavefront", "stencil_wavefront_info",
+                    "model_predict_wavefront"]

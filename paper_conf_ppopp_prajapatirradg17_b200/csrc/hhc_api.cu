@@ -530,6 +530,72 @@ extern "C" int stencil_run_host(stencil_t h, const float* h_in, float* h_out, in
     return cuda_fail(h, cudaStreamSynchronize(s));
 }
 
+// ---- wavefront-parallel Jacobi-1D (reading W1)
+static int check_wave_tile(stencil_tile t) {
+    if (t.t < 1 || t.t > 1024 || t.s1 < 2 || t.s1 > 16384) return STENCIL_ETILE;
+    return STENCIL_OK;
+}
+
+extern "C" int stencil_wavefront_info(const int64_t* dims, int64_t T, stencil_tile tile, int64_t* n_wavefronts,
+                                      int64_t* n_tiles, int64_t* max_width) {
+    if (!dims || dims[0] < 3 || T < 1) return STENCIL_EINVAL;
+    if (int rc = check_wave_tile(tile)) return rc;
+    std::vector<WaveLaunch> ws;
+    wave1d_schedule(dims[0], T, tile.t, tile.s1, ws);
+    int64_t tiles = 0, mx = 0;
+    for (auto& w : ws) { tiles += w.n; mx = std::max(mx, w.n); }
+    if (n_wavefronts) *n_wavefronts = (int64_t)ws.size();
+    if (n_tiles) *n_tiles = tiles;
+    if (max_width) *max_width = mx;
+    return STENCIL_OK;
+}
+
+extern "C" int stencil_run_wavefront(stencil_t h, const float* d_in, float* d_out, int64_t T, stencil_tile tile,
+                                     void* cuda_stream) {
+    if (!h) return STENCIL_EINVAL;
+    if (h->sticky) return h->sticky;
+    if (h->kind != STENCIL_JACOBI1D_3PT || h->ndims != 1) return STENCIL_EINVAL;
+    if (!d_in || !d_out || T < 0) return STENCIL_EINVAL;
+    const int64_t n = h->nelem();
+    if (d_out < d_in + n && d_in < d_out + n) return STENCIL_EINVAL;
+    cudaStream_t s = (cudaStream_t)cuda_stream;
+    cudaSetDevice(h->device);
+    if (T == 0) {
+        h->last_launches = 1;
+        launch_copy_full(d_in, d_out, n, s);
+        return cuda_fail(h, cudaGetLastError());
+    }
+    if (int rc = check_wave_tile(tile)) return rc;
+    if (wave1d_smem_bytes(tile.t, tile.s1) > h->smem_optin) return STENCIL_ETILE;
+    if (!h->scratch) {
+        cudaError_t e = cudaMalloc(&h->scratch, n * sizeof(float));
+        if (e != cudaSuccess) { h->scratch = nullptr; return STENCIL_ENOMEM; }
+    }
+    float* plane[2];
+    plane[T & 1] = d_out;
+    plane[1 - (T & 1)] = h->scratch;
+    launch_copy_full(d_in, plane[0], n, s);                 // a2: level 0 in plane 0
+    launch_copy_ring(d_in, plane[1], n, 1, 1, s);           // the two ring points in plane 1
+    std::vector<WaveLaunch> ws;
+    wave1d_schedule(n, T, tile.t, tile.s1, ws);
+    WaveParams p;
+    memset(&p, 0, sizeof(p));
+    p.plane[0] = plane[0];
+    p.plane[1] = plane[1];
+    p.S = n; p.T = T; p.tT = tile.t; p.tS = tile.s1;
+    for (int k = 0; k < 3; ++k) p.w[k] = h->w[k];
+    p.c = h->c;
+    for (auto& w : ws) {
+        p.d = w.d; p.ia = w.ia;
+        if (launch_wave1d(h->mode, h->has_c, h->defw, p, w.n, s)) {
+            h->sticky = STENCIL_ECUDA;
+            return STENCIL_ECUDA;
+        }
+    }
+    h->last_launches = 2 + (int64_t)ws.size();
+    return cuda_fail(h, cudaGetLastError());
+}
+
 extern "C" int64_t stencil_last_launches(stencil_t h) { return h ? h->last_launches : 0; }
 
 extern "C" int stencil_profile(stencil_t h, const float* d_in, float* d_out, int64_t T, stencil_tile tile,

@@ -2,6 +2,8 @@
 // files (never by the oracle).  See DESIGN.md §Kernels for the layouts.
 #pragma once
 #include <stdint.h>
+#include <algorithm>
+#include <vector>
 
 #include "../../include/hhc.h"
 
@@ -60,6 +62,41 @@ void launch_copy_ring(const float* in, float* out, int64_t S1, int64_t S2, int64
 void launch_copy_full(const float* in, float* out, int64_t n, void* stream);
 
 void set_compute_only(stencil_t h, int on);
+
+// ---- wavefront-parallel Jacobi-1D (reading W1)
+// Parallelogram tiles in skewed coordinates x' = x + t: tile (i, j) computes the
+// levels t in (i*tT, min((i+1)*tT, T)] at x' in [j*tS, (j+1)*tS).  Wavefront d
+// holds the tiles with i + j = d that contain an interior point; they are
+// independent (one launch per wavefront) and form a contiguous i range.
+struct WaveLaunch {
+    int64_t d, ia, n;      // tiles i = ia .. ia+n-1, j = d - i
+    int nlev_max;          // levels of the tallest tile of the wavefront
+};
+inline void wave1d_schedule(int64_t S, int64_t T, int tT, int tS, std::vector<WaveLaunch>& out) {
+    out.clear();
+    const int64_t n = S - 2, Nt = (T + tT - 1) / tT;
+    if (n <= 0 || T <= 0) return;
+    auto jlo = [&](int64_t i) { return (1 + i * tT + 1) / tS; };
+    auto jhi = [&](int64_t i) { return (n + std::min<int64_t>((i + 1) * tT, T)) / tS; };
+    const int64_t dmin = jlo(0), dmax = Nt - 1 + jhi(Nt - 1);
+    int64_t ia = 0, ib = -1;
+    for (int64_t d = dmin; d <= dmax; ++d) {
+        while (ia < Nt && ia + jhi(ia) < d) ++ia;             // suffix: i + jhi(i) >= d
+        while (ib + 1 < Nt && ib + 1 + jlo(ib + 1) <= d) ++ib;  // prefix: i + jlo(i) <= d
+        if (ia > ib) continue;
+        const int64_t last = std::min<int64_t>(tT, T - ib * tT);
+        out.push_back(WaveLaunch{d, ia, ib - ia + 1, ib > ia ? tT : (int)last});
+    }
+}
+inline int64_t wave1d_smem_bytes(int tT, int tS) { return 4 * (2 * ((int64_t)tS + 2) + 2 * (int64_t)tT + 2); }
+
+struct WaveParams {
+    float* plane[2];       // plane[t & 1] holds level t (ring in both)
+    int64_t S, T, d, ia;
+    int tT, tS;
+    float w[3], c;
+};
+int launch_wave1d(int mode, bool has_c, bool defw, const WaveParams& p, int64_t nblocks, void* stream);
 
 // Microbenchmarks (microbench.cu)
 int run_microbench(int which, int kind, int ndims, const int64_t* dims, int64_t T,

@@ -211,6 +211,52 @@ extern "C" double model_predict(stencil_kind kind, int ndims, const int64_t* dim
     return f(ndims, S, T, tile, *hw);
 }
 
+// Wavefront-parallel Jacobi-1D: "the total execution time is
+// the sum of the times for each wavefront ... equation 6 holds for wavefront
+// parallel codes".  Eq. 6 per wavefront d of n_d parallelogram
+// tiles: T_sync + ceil(ceil(n_d/k)/nSM) * Ttile, Ttile by Eq. 10 (k = 1) or
+// Eq. 12 (k > 1) with Eq. 8's m' = (mi + mo) L + 2 tau_sync and Eq. 9's
+// c = sum over the tile's rows of C_iter ceil(tS/nV) + tau_sync.  Footprint of a
+// tile of nlev levels (reading W1): mi = tS + 2 + 2(nlev-1) words in
+// (bottom row + left halo), mo = tS + 2(nlev-1) out (top row + right edge).
+extern "C" double model_predict_wavefront(stencil_kind kind, int ndims, const int64_t* dims, int64_t T,
+                                          stencil_tile tile, const model_hw_params* hw) {
+    const double nan = std::numeric_limits<double>::quiet_NaN();
+    if (!hw || !dims || kind != STENCIL_JACOBI1D_3PT || ndims != 1 || T < 1 || dims[0] < 3) return nan;
+    if (tile.t < 1 || tile.s1 < 2) return nan;
+    if (hw->n_sm < 1 || hw->n_v < 1 || hw->mtb_sm < 1 || hw->m_sm_bytes < 1 || hw->m_block_bytes < 1) return nan;
+    const double inf = std::numeric_limits<double>::infinity();
+    const int64_t tS = tile.s1;
+    const int64_t Mtile = hhc::wave1d_smem_bytes(tile.t, tile.s1);
+    if (Mtile > hw->m_block_bytes) return inf;
+    int64_t k = std::min<int64_t>(hw->m_sm_bytes / Mtile, hw->mtb_sm);         // Eq. 11
+    if (hw->geometry == 1) {
+        k = std::min<int64_t>(k, (hw->max_threads_sm > 0 ? hw->max_threads_sm : 2048) / 256);
+        if (hw->regs_per_thread > 0) k = std::min<int64_t>(k, hw->r_sm / (hw->regs_per_thread * 256));
+    }
+    if (k < 1) return inf;
+    const double L = hw->geometry == 1 ? hw->L_s_per_word * hw->n_sm : hw->L_s_per_word;   // reading M5
+    std::vector<hhc::WaveLaunch> ws;
+    hhc::wave1d_schedule(dims[0], T, tile.t, tile.s1, ws);
+    double total = 0.0;
+    for (const auto& w : ws) {
+        const int64_t nl = w.nlev_max;
+        const double mi = (double)(tS + 2 + 2 * (nl - 1)), mo = (double)(tS + 2 * (nl - 1));
+        const double m_prime = (mi + mo) * L + 2.0 * hw->tau_sync_s;                      // Eq. 8
+        const double c = (double)nl * (hw->C_iter_s * (double)cdiv(tS, hw->n_v) + hw->tau_sync_s);   // Eq. 9
+        if (hw->geometry == 1) {
+            // reading W2: the busiest SM holds ceil(n_d / nSM) tiles (round-robin), min(k, that) at a time
+            const int64_t m = cdiv(w.n, hw->n_sm), ke = std::min(k, m);
+            const double Ttile = ke == 1 ? m_prime + c : m_prime + c + (double)(ke - 1) * std::max(m_prime, c);
+            total += hw->T_sync_s + Ttile * (double)cdiv(m, ke);
+        } else {
+            const double Ttile = k == 1 ? m_prime + c : m_prime + c + (double)(k - 1) * std::max(m_prime, c);   // Eq. 10/12
+            total += hw->T_sync_s + Ttile * (double)cdiv(cdiv(w.n, k), hw->n_sm);            // Eq. 6
+        }
+    }
+    return total;
+}
+
 extern "C" int model_select_tile(stencil_kind kind, int ndims, const int64_t* dims, int64_t T,
                                  const model_hw_params* hw, double within, stencil_tile* best, int* best_threads,
                                  stencil_tile* cands, int cap, int* n_cands) {

@@ -397,3 +397,44 @@ def test_overlapped_slabs_gpu_streams(kind, dims, T, tT, world):
     for r in range(world):
         lo, hi, got = out[r]
         assert_bits(np.ascontiguousarray(got), np.ascontiguousarray(exp[lo:hi]), f"rank {r}")
+
+
+# ---- wavefront-parallel Jacobi-1D (reading W1): K3, one block per
+# parallelogram tile, one launch per wavefront; the same oracle as every other schedule
+def gpu_run_wavefront(a, T, tile, mode=hhc.FUSED, coeffs=None):
+    s = hhc.stencil_create(hhc.JACOBI1D_3PT, a.shape, coeffs=coeffs, mode=mode)
+    d_in = torch.from_numpy(np.ascontiguousarray(a)).to(DEV)
+    d_out = torch.full_like(d_in, float("nan"))
+    hhc.stencil_run_wavefront(s, d_in, d_out, T, tile)
+    torch.cuda.synchronize()
+    nw = hhc.stencil_wavefront_info(a.shape, T, tile)[0] if T > 0 else 0
+    assert hhc.stencil_last_launches(s) == (2 + nw if T > 0 else 1)
+    res = d_out.cpu().numpy()
+    assert np.array_equal(d_in.cpu().numpy().view(np.uint32), a.view(np.uint32))   # in untouched
+    hhc.stencil_destroy(s)
+    return res
+
+
+@pytest.mark.parametrize("mode", [hhc.PLAIN, hhc.FUSED])
+def test_parity_wavefront_1d(mode):
+    rng = np.random.default_rng(90 + mode)
+    for tile in [(1, 2), (2, 3), (3, 7), (8, 32), (16, 256), (5, 1000), (64, 4096)]:
+        n = int(rng.integers(3, 6000))
+        a = field(int(rng.integers(1, 1 << 30)), (n,))
+        for T in (0, 1, 2, 7, tile[0] + 1, 3 * tile[0] + 5):
+            exp = oracle.run(hhc.JACOBI1D_3PT, a, T, mode)
+            got = gpu_run_wavefront(a, T, tile, mode)
+            assert_bits(got, exp, f"wavefront n {n} T {T} tile {tile}")
+
+
+def test_parity_wavefront_1d_large_and_coeffs():
+    a = field(91, (400_003,))
+    for T, tile in ((64, (16, 2048)), (37, (4, 8192)), (100, (100, 1024))):
+        assert_bits(gpu_run_wavefront(a, T, tile), oracle.run(hhc.JACOBI1D_3PT, a, T, hhc.FUSED),
+                    f"wavefront large T {T} tile {tile}")
+    coeffs = [0.25, 0.5, 0.25, 0.001]
+    for mode in (hhc.PLAIN, hhc.FUSED):
+        assert_bits(gpu_run_wavefront(a[:20001], 33, (8, 256), mode, coeffs=coeffs),
+                    oracle.run(hhc.JACOBI1D_3PT, a[:20001], 33, mode, coeffs=coeffs), "wavefront coeffs")
+    # the two schedules of the same update agree bit for bit
+    assert_bits(gpu_run_wavefront(a, 50, (10, 512)), gpu_run(hhc.JACOBI1D_3PT, a, 50, (16, 2048)), "wave vs hex")
