@@ -188,8 +188,9 @@ int stencil_profile(stencil_t h, const float* d_in, float* d_out, int64_t T, ste
 
 /* A_T from A_0 like stencil_run (same pointer rules, stream-ordered,
  * asynchronous, scratch plane owned by the handle), on a handle created for
- * STENCIL_JACOBI1D_3PT (else STENCIL_EINVAL).  Not graph-captured: one launch
- * per wavefront plus two set-up copies. */
+ * STENCIL_JACOBI1D_3PT (else STENCIL_EINVAL).  One launch per wavefront plus
+ * two set-up copies, captured once into a CUDA graph per (pointers, T, tile)
+ * and replayed, like stencil_run. */
 int stencil_run_wavefront(stencil_t h, const float* d_in, float* d_out, int64_t T,
                           stencil_tile tile, void* cuda_stream);
 

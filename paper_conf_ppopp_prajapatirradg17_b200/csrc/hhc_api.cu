@@ -391,7 +391,10 @@ static int enqueue_rows(stencil_t h, const int64_t* dims, const float* ring, flo
     return STENCIL_OK;
 }
 
+static int enqueue_wavefront(stencil_t h, const RunSpec& r, cudaStream_t s, int64_t* launches);
+
 static int enqueue_spec(stencil_t h, const RunSpec& r, cudaStream_t s, int64_t* launches) {
+    if (r.planes_mode == 2) return enqueue_wavefront(h, r, s, launches);
     const int64_t n = r.dims[0] * r.dims[1] * r.dims[2];
     int64_t nl = 0, nrows = 0;
     int rc;
@@ -421,7 +424,7 @@ static bool same_spec(const RunSpec& x, const RunSpec& y) {
 
 // Run a spec through the CUDA-graph cache (captured once per spec, replayed).
 static int run_spec(stencil_t h, const RunSpec& r, cudaStream_t s) {
-    int prc = prepare_rows(h, r.dims, r.T, r.tile, r.thr, r.nr);
+    int prc = r.planes_mode == 2 ? STENCIL_OK : prepare_rows(h, r.dims, r.T, r.tile, r.thr, r.nr);
     if (prc) return prc;
     const bool use_graph = getenv("HHC_NO_GRAPH") == nullptr && !h->compute_only;
     if (!use_graph) {
@@ -550,6 +553,30 @@ extern "C" int stencil_wavefront_info(const int64_t* dims, int64_t T, stencil_ti
     return STENCIL_OK;
 }
 
+static int enqueue_wavefront(stencil_t h, const RunSpec& r, cudaStream_t s, int64_t* launches) {
+    const int64_t n = r.dims[0];
+    float* plane[2];
+    plane[r.T & 1] = r.b;
+    plane[1 - (r.T & 1)] = h->scratch;
+    launch_copy_full(r.a, plane[0], n, s);                  // a2: level 0 in plane 0
+    launch_copy_ring(r.a, plane[1], n, 1, 1, s);            // the two ring points in plane 1
+    std::vector<WaveLaunch> ws;
+    wave1d_schedule(n, r.T, r.tile.t, r.tile.s1, ws);
+    WaveParams p;
+    memset(&p, 0, sizeof(p));
+    p.plane[0] = plane[0];
+    p.plane[1] = plane[1];
+    p.S = n; p.T = r.T; p.tT = r.tile.t; p.tS = r.tile.s1;
+    for (int k = 0; k < 3; ++k) p.w[k] = h->w[k];
+    p.c = h->c;
+    for (auto& w : ws) {
+        p.d = w.d; p.ia = w.ia;
+        if (launch_wave1d(h->mode, h->has_c, h->defw, p, w.n, s)) return cuda_fail(h, cudaErrorLaunchFailure);
+    }
+    *launches = 2 + (int64_t)ws.size();
+    return STENCIL_OK;
+}
+
 extern "C" int stencil_run_wavefront(stencil_t h, const float* d_in, float* d_out, int64_t T, stencil_tile tile,
                                      void* cuda_stream) {
     if (!h) return STENCIL_EINVAL;
@@ -571,29 +598,15 @@ extern "C" int stencil_run_wavefront(stencil_t h, const float* d_in, float* d_ou
         cudaError_t e = cudaMalloc(&h->scratch, n * sizeof(float));
         if (e != cudaSuccess) { h->scratch = nullptr; return STENCIL_ENOMEM; }
     }
-    float* plane[2];
-    plane[T & 1] = d_out;
-    plane[1 - (T & 1)] = h->scratch;
-    launch_copy_full(d_in, plane[0], n, s);                 // a2: level 0 in plane 0
-    launch_copy_ring(d_in, plane[1], n, 1, 1, s);           // the two ring points in plane 1
-    std::vector<WaveLaunch> ws;
-    wave1d_schedule(n, T, tile.t, tile.s1, ws);
-    WaveParams p;
-    memset(&p, 0, sizeof(p));
-    p.plane[0] = plane[0];
-    p.plane[1] = plane[1];
-    p.S = n; p.T = T; p.tT = tile.t; p.tS = tile.s1;
-    for (int k = 0; k < 3; ++k) p.w[k] = h->w[k];
-    p.c = h->c;
-    for (auto& w : ws) {
-        p.d = w.d; p.ia = w.ia;
-        if (launch_wave1d(h->mode, h->has_c, h->defw, p, w.n, s)) {
-            h->sticky = STENCIL_ECUDA;
-            return STENCIL_ECUDA;
-        }
-    }
-    h->last_launches = 2 + (int64_t)ws.size();
-    return cuda_fail(h, cudaGetLastError());
+    if (prepare_wave1d(h->mode, h->has_c, h->defw, tile.t, tile.s1)) return cuda_fail(h, cudaErrorInvalidValue);
+    // through the CUDA-graph cache like stencil_run (one graph per pointers/T/tile)
+    RunSpec r;
+    memset(&r, 0, sizeof(r));
+    r.planes_mode = 2; r.a = d_in; r.b = d_out;
+    r.dims[0] = n; r.dims[1] = 1; r.dims[2] = 1;
+    r.T = T; r.tile = tile; r.tile.s2 = r.tile.s3 = 0;
+    r.G = 1; r.thr = 256; r.nr = 0;
+    return run_spec(h, r, s);
 }
 
 extern "C" int64_t stencil_last_launches(stencil_t h) { return h ? h->last_launches : 0; }

@@ -88,7 +88,8 @@ inline void wave1d_schedule(int64_t S, int64_t T, int tT, int tS, std::vector<Wa
         out.push_back(WaveLaunch{d, ia, ib - ia + 1, ib > ia ? tT : (int)last});
     }
 }
-inline int64_t wave1d_smem_bytes(int tT, int tS) { return 4 * (2 * ((int64_t)tS + 2) + 2 * (int64_t)tT + 2); }
+// two level rows of tS + 2 slots, each padded to 16 B with slot 2 aligned, + the halo table
+inline int64_t wave1d_smem_bytes(int tT, int tS) { return 4 * (2 * (((int64_t)tS + 4 + 3) & ~3) + 2 * (int64_t)tT); }
 
 struct WaveParams {
     float* plane[2];       // plane[t & 1] holds level t (ring in both)
@@ -97,6 +98,7 @@ struct WaveParams {
     float w[3], c;
 };
 int launch_wave1d(int mode, bool has_c, bool defw, const WaveParams& p, int64_t nblocks, void* stream);
+int prepare_wave1d(int mode, bool has_c, bool defw, int tT, int tS);
 
 // Microbenchmarks (microbench.cu)
 int run_microbench(int which, int kind, int ndims, const int64_t* dims, int64_t T,

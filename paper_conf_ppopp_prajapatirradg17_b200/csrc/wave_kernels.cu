@@ -23,14 +23,19 @@
 
 namespace hhc {
 
-template <int MODE, bool HASC, bool DEFW>
+// VEC (tS % 4 == 0): each thread computes aligned groups of 4 slots (one LDS.128 + one
+// LDS.64 of the level below, one STS.128), with a branch-free body when the whole
+// level lies inside the interior; rows start 2 floats into a 16-B line so that
+// slot 2 (the tile's first own column) is 16-B aligned.
+template <int MODE, bool HASC, bool DEFW, bool VEC>
 __global__ void __launch_bounds__(256) wave1d_kernel(const __grid_constant__ WaveParams p) {
     extern __shared__ __align__(16) float smw[];
     const int tS = p.tS, tT = p.tT;
     const int RW = tS + 2;                                   // slots k: x' = j*tS - 2 + k
-    float* const buf0 = smw;
-    float* const buf1 = smw + RW;
-    float* const halo = smw + 2 * RW;                        // [tT][2]: columns k = 0, 1 of level t0 + l
+    const int RWP = (RW + 2 + 3) & ~3;                       // padded row: slot k at row[2 + k]
+    float* const buf0 = smw + 2;
+    float* const buf1 = smw + RWP + 2;
+    float* const halo = smw + 2 * RWP;                       // [tT][2]: columns k = 0, 1 of level t0 + l
     const int nthr = blockDim.x, tid = threadIdx.x;
     const int64_t i = p.ia + blockIdx.x, j = p.d - i;
     const int64_t t0 = i * tT;                               // input level of the band
@@ -74,6 +79,28 @@ __global__ void __launch_bounds__(256) wave1d_kernel(const __grid_constant__ Wav
         float* const dst = p.plane[t & 1];
         if (tid < 2 && l < nlev) cur[tid] = halo[2 * l + tid];
         const bool top = l == nlev;
+        if constexpr (VEC) {
+            // slots 2 .. RW-1 in aligned groups of 4; x of slot k is xb + k - t
+            const int64_t xlo = xb + 2 - t, xhi = xb + RW - 1 - t;
+            if (xlo >= 1 && xhi <= S - 2) {                      // the whole level is interior
+                for (int k = 2 + 4 * tid; k < RW; k += 4 * nthr) {
+                    const float2 lo = *reinterpret_cast<const float2*>(prev + k - 2);
+                    const float4 v = *reinterpret_cast<const float4*>(prev + k);
+                    const float4 o = make_float4(pt(lo.x, lo.y, v.x), pt(lo.y, v.x, v.y), pt(v.x, v.y, v.z),
+                                                 pt(v.y, v.z, v.w));
+                    *reinterpret_cast<float4*>(cur + k) = o;
+                    if (top) {
+                        float* g = dst + (xb + k - t);
+                        g[0] = o.x; g[1] = o.y; g[2] = o.z; g[3] = o.w;
+                    } else if (k + 4 >= RW) {                    // the group holding slots tS, tS+1
+                        dst[xb + tS - t] = o.z;
+                        dst[xb + tS + 1 - t] = o.w;
+                    }
+                }
+                __syncthreads();
+                continue;
+            }
+        }
         for (int k = 2 + tid; k < RW; k += nthr) {
             const int64_t x = xb + k - t;
             // interior: Eq. 1; the ring (x = 0, S-1) keeps its value, which sits
@@ -87,20 +114,33 @@ __global__ void __launch_bounds__(256) wave1d_kernel(const __grid_constant__ Wav
     }
 }
 
-int launch_wave1d(int mode, bool has_c, bool defw, const WaveParams& p, int64_t nblocks, void* stream) {
+static void (*pick_wave1d(int mode, bool has_c, bool defw, bool vec))(WaveParams) {
     void (*k)(WaveParams);
-    if (mode == STENCIL_MODE_FUSED)
-        k = defw ? wave1d_kernel<1, false, true> : has_c ? wave1d_kernel<1, true, false> : wave1d_kernel<1, false, false>;
-    else
-        k = defw ? wave1d_kernel<0, false, true> : has_c ? wave1d_kernel<0, true, false> : wave1d_kernel<0, false, false>;
-    const int64_t smem = wave1d_smem_bytes(p.tT, p.tS);
-    static int64_t set_smem[2][3] = {};
-    const int vi = defw ? 0 : has_c ? 1 : 2;
-    if (smem > 48 * 1024 && smem > set_smem[mode][vi]) {
-        cudaError_t e = cudaFuncSetAttribute((const void*)k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        if (e != cudaSuccess) return STENCIL_ECUDA;
-        set_smem[mode][vi] = smem;
+    if (vec) {
+        if (mode == STENCIL_MODE_FUSED)
+            k = defw ? wave1d_kernel<1, false, true, true> : has_c ? wave1d_kernel<1, true, false, true> : wave1d_kernel<1, false, false, true>;
+        else
+            k = defw ? wave1d_kernel<0, false, true, true> : has_c ? wave1d_kernel<0, true, false, true> : wave1d_kernel<0, false, false, true>;
+    } else {
+        if (mode == STENCIL_MODE_FUSED)
+            k = defw ? wave1d_kernel<1, false, true, false> : has_c ? wave1d_kernel<1, true, false, false> : wave1d_kernel<1, false, false, false>;
+        else
+            k = defw ? wave1d_kernel<0, false, true, false> : has_c ? wave1d_kernel<0, true, false, false> : wave1d_kernel<0, false, false, false>;
     }
+    return k;
+}
+
+// the kernel's dynamic shared-memory limit, set outside any stream capture
+int prepare_wave1d(int mode, bool has_c, bool defw, int tT, int tS) {
+    auto k = pick_wave1d(mode, has_c, defw, tS % 4 == 0);
+    const int64_t smem = wave1d_smem_bytes(tT, tS);
+    cudaError_t e = cudaFuncSetAttribute((const void*)k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    return e == cudaSuccess ? STENCIL_OK : STENCIL_ECUDA;
+}
+
+int launch_wave1d(int mode, bool has_c, bool defw, const WaveParams& p, int64_t nblocks, void* stream) {
+    auto k = pick_wave1d(mode, has_c, defw, p.tS % 4 == 0);
+    const int64_t smem = wave1d_smem_bytes(p.tT, p.tS);
     void* args[] = {const_cast<WaveParams*>(&p)};
     cudaError_t e = cudaLaunchKernel((const void*)k, dim3((unsigned)nblocks), dim3(256), args, (size_t)smem,
                                      (cudaStream_t)stream);
