@@ -42,6 +42,9 @@ CONFIGS = {
     # SURVEY §8(f) f2 (not a BASELINE.json config): the paper's 1D derivation case
     "X1": dict(kind=7, dims=(1 << 26,), T=1024, tile=(128, 2048), threads=256,
                desc="Jacobi-1D 3-point fp32, 2^26 points, T=1024 (extension f2)"),
+    # SURVEY §8(f) f3 (not a BASELINE.json config): the wavefront-parallel schedule
+    "W1": dict(kind=7, dims=((1 << 22) + 2,), T=1024, tile=(4, 8192), threads=256, schedule="wavefront",
+               desc="Jacobi-1D 3-point fp32, 2^22 interior points, T=1024, wavefront schedule (extension f3)"),
 }
 DEFAULT_CONFIG = "C2"
 
@@ -241,8 +244,16 @@ def bench_single(args, cfg, cfgname):
     s = hhc.stencil_create(kind, dims, mode=mode)
     stream = torch.cuda.current_stream()
 
+    wave = cfg.get("schedule") == "wavefront"
+
+    def run(a, b):
+        if wave:
+            hhc.stencil_run_wavefront(s, a, b, T, tile, stream)
+        else:
+            hhc.stencil_run(s, a, b, T, tile, threads, stream)
+
     for _ in range(args.warmup):
-        hhc.stencil_run(s, d_in, d_out, T, tile, threads, stream)
+        run(d_in, d_out)
     torch.cuda.synchronize()
     launches_per_step = hhc.stencil_last_launches(s)
 
@@ -253,7 +264,7 @@ def bench_single(args, cfg, cfgname):
     torch.cuda.synchronize()
     e0.record(stream)
     for _ in range(args.steps):
-        hhc.stencil_run(s, d_in, d_out, T, tile, threads, stream)
+        run(d_in, d_out)
     e1.record(stream)
     torch.cuda.synchronize()
     clocks = sampler.stop()
@@ -262,7 +273,12 @@ def bench_single(args, cfg, cfgname):
     value = n_upd * args.steps / dt / 1e9
 
     # dominant kernel: per-launch device time of the HHC rows (events on the launching stream)
-    ksec, klaunch = hhc.stencil_profile(s, d_in, d_out, T, tile, threads, stream)
+    if wave:
+        # the wavefront launches are one CUDA graph with the two set-up copies (16 MB each, < 1 % of the
+        # step): the kernel time is the step time
+        ksec, klaunch = dt / args.steps, launches_per_step - 2
+    else:
+        ksec, klaunch = hhc.stencil_profile(s, d_in, d_out, T, tile, threads, stream)
     flops = FLOPS_PER_UPDATE[kind] * n_upd
     peaks = load_peaks()
     peak = fp32_peak_tflops(peaks)
@@ -270,7 +286,7 @@ def bench_single(args, cfg, cfgname):
     traffic = ncu_traffic(cfgname)
     roofline = {"bound": "alu", "achieved": round(achieved, 3), "peak": round(peak, 2), "unit": "TFLOP/s",
                 "frac": round(achieved / peak, 4), "traffic": traffic,
-                "kernel": {1: "hex1d_kernel", 2: "hex2d_kernel", 3: "hex3d_kernel"}[len(dims)],
+                "kernel": "wave1d_kernel" if wave else {1: "hex1d_kernel", 2: "hex2d_kernel", 3: "hex3d_kernel"}[len(dims)],
                 "kernel_share_of_step": round(ksec / (dt / args.steps), 4),
                 "kernel_launches_per_step": klaunch,
                 "peak_basis": "148 SM x 128 FP32 lanes x 2 x sm_max_mhz (MEASURED_PEAKS.json)"}
@@ -278,11 +294,20 @@ def bench_single(args, cfg, cfgname):
     e2e = None
     if not args.no_e2e:
         h_out = torch.empty_like(h_in).pin_memory()
-        hhc.stencil_run_host(s, h_in, h_out, T, tile, threads, stream)
+
+        def run_host():
+            if wave:     # pinned host -> device, run, device -> host, synchronise
+                d_in.copy_(h_in, non_blocking=True)
+                run(d_in, d_out)
+                h_out.copy_(d_out, non_blocking=True)
+                torch.cuda.synchronize()
+            else:
+                hhc.stencil_run_host(s, h_in, h_out, T, tile, threads, stream)
+        run_host()
         torch.cuda.synchronize()
         t0 = time.perf_counter()
         for _ in range(args.steps):
-            hhc.stencil_run_host(s, h_in, h_out, T, tile, threads, stream)
+            run_host()
         et = time.perf_counter() - t0
         nbytes = host.nbytes
         e2e = {"value": n_upd * args.steps / et / 1e9, "unit": METRIC, "h2d_bytes_per_step": nbytes,
@@ -298,8 +323,12 @@ def bench_single(args, cfg, cfgname):
         "config": {"workload": cfgname + ": " + cfg["desc"], "tile": list(tile), "threads": threads,
                    "mode": args.mode, "updates_per_step": n_upd,
                    "l2": "inputs larger than L2 (plane %d MB > 126 MB)" % (host.nbytes >> 20)
-                   if host.nbytes > 126e6 else "inputs smaller than L2 (launch-bound config)",
-                   "parallelism": "1 GPU, one CTA per hexagonal prism"},
+                   if host.nbytes > 126e6 else ("planes of %d MB stay in L2, not flushed (extension config: "
+                                                "each wavefront re-reads rows the previous launch wrote)"
+                                                % (host.nbytes >> 20) if wave
+                                                else "inputs smaller than L2 (launch-bound config)"),
+                   "parallelism": "1 GPU, one CTA per parallelogram tile, one launch per wavefront" if wave
+                   else "1 GPU, one CTA per hexagonal prism"},
         "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
         "gpu_launches": launches_per_step * args.steps,
     }

@@ -46,9 +46,16 @@ __global__ void __launch_bounds__(256) wave1d_kernel(const __grid_constant__ Wav
     const float w0 = DEFW ? third : p.w[0], w1 = DEFW ? third : p.w[1], w2 = DEFW ? third : p.w[2];
     {
         const float* src = p.plane[t0 & 1];
-        for (int k = tid; k < RW; k += nthr) {
-            const int64_t x = xb + k - t0;
-            buf0[k] = (x >= 0 && x < S) ? __ldcg(src + x) : 0.0f;
+        const int64_t x0 = xb - t0;                          // x of slot 0 at level t0
+        if (x0 >= 0 && x0 + RW <= S) {                       // the whole bottom row is in the array:
+            const float* s0 = src + x0;                      // unchecked, unrolled for loads in flight
+#pragma unroll 8
+            for (int k = tid; k < RW; k += nthr) buf0[k] = __ldcg(s0 + k);
+        } else {
+            for (int k = tid; k < RW; k += nthr) {
+                const int64_t x = x0 + k;
+                buf0[k] = (x >= 0 && x < S) ? __ldcg(src + x) : 0.0f;
+            }
         }
         for (int e = tid; e < 2 * (nlev - 1); e += nthr) {
             const int l = 1 + (e >> 1), k = e & 1;
