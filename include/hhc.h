@@ -207,6 +207,16 @@ int stencil_wavefront_info(const int64_t* dims, int64_t T, stencil_tile tile,
 double model_predict_wavefront(stencil_kind kind, int ndims, const int64_t* dims, int64_t T,
                                stencil_tile tile, const model_hw_params* hw);
 
+/* Eq. 31 for the wavefront schedule (reading W3): *best = argmin of
+ * model_predict_wavefront over t in [1, min(T, 128)] and s1 in {4, 6, 8, 12,
+ * 16, 24, ...} (powers of two and 1.5x) up to min(16384, S + T rounded up to 4);
+ * ties -> smallest (t, s1).  Tiles with Talg <= (1+within) Talg_min go to
+ * cands[0..min(n, cap)) in enumeration order (t outer), *n_cands = n.
+ * STENCIL_EINVAL for bad arguments, STENCIL_ETILE if nothing fits. */
+int model_select_wavefront_tile(stencil_kind kind, int ndims, const int64_t* dims, int64_t T,
+                                const model_hw_params* hw, double within, stencil_tile* best,
+                                stencil_tile* cands, int cap, int* n_cands);
+
 /* Human-readable status. */
 const char* stencil_strerror(int status);
 

@@ -120,6 +120,9 @@ def load(build_if_missing: bool = False):
     lib.model_predict_wavefront.argtypes = [ctypes.c_int, ctypes.c_int, i64p, ctypes.c_int64, stencil_tile,
                                             P(model_hw_params)]
     lib.model_predict_wavefront.restype = ctypes.c_double
+    lib.model_select_wavefront_tile.argtypes = [ctypes.c_int, ctypes.c_int, i64p, ctypes.c_int64,
+                                                P(model_hw_params), ctypes.c_double, P(stencil_tile),
+                                                P(stencil_tile), ctypes.c_int, P(ctypes.c_int)]
     _lib = lib
     return lib
 
@@ -241,6 +244,18 @@ def model_predict_wavefront(dims, T: int, tile, hw: model_hw_params) -> float:
     return float(load().model_predict_wavefront(JACOBI1D_3PT, nd, d, int(T), make_tile(tile), ctypes.byref(hw)))
 
 
+def model_select_wavefront_tile(dims, T: int, hw: model_hw_params, within: float = 0.10, cap: int = 10000):
+    """(best (t, s1), candidate (t, s1) list) for the wavefront schedule."""
+    d, nd = _dims(dims)
+    best = stencil_tile()
+    cands = (stencil_tile * cap)()
+    n = ctypes.c_int()
+    _check(load().model_select_wavefront_tile(JACOBI1D_3PT, nd, d, int(T), ctypes.byref(hw), float(within),
+                                              ctypes.byref(best), cands, cap, ctypes.byref(n)),
+           "model_select_wavefront_tile")
+    return best.astuple()[:2], [cands[i].astuple()[:2] for i in range(min(n.value, cap))]
+
+
 def stencil_last_launches(s: Stencil) -> int:
     return int(load().stencil_last_launches(s.handle))
 
@@ -298,4 +313,4 @@ EXPORTED_SYMBOLS = ["stencil_create", "stencil_destroy", "stencil_run", "stencil
                     "stencil_run_planes", "model_predict", "model_select_tile", "stencil_tile_resources",
                     "stencil_plan_info", "stencil_microbench", "stencil_strerror", "stencil_last_launches",
                     "stencil_profile", "stencil_run_wavefront", "stencil_wavefront_info",
-                    "model_predict_wavefront"]
+                    "model_predict_wavefront", "model_select_wavefront_tile"]

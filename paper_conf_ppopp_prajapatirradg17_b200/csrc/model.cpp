@@ -257,6 +257,46 @@ extern "C" double model_predict_wavefront(stencil_kind kind, int ndims, const in
     return total;
 }
 
+// The wavefront schedule's tile by exhaustive enumeration of Talg (Eq. 31's
+// argmin, on model_predict_wavefront; reading W3):
+// tT in [1, min(T, 128)], tS in {4, 6, 8, 12, 16, ..., 2^k, 1.5 * 2^k, ...} up to
+// min(16384, the 4-rounded S + T); ties -> the smallest (t, s1).
+extern "C" int model_select_wavefront_tile(stencil_kind kind, int ndims, const int64_t* dims, int64_t T,
+                                           const model_hw_params* hw, double within, stencil_tile* best,
+                                           stencil_tile* cands, int cap, int* n_cands) {
+    if (!hw || !dims || !best || kind != STENCIL_JACOBI1D_3PT || ndims != 1 || T < 1 || dims[0] < 3 || within < 0)
+        return STENCIL_EINVAL;
+    std::vector<int> tss;
+    const int64_t smax = std::min<int64_t>(16384, ((dims[0] - 2 + T) + 3) / 4 * 4);
+    for (int64_t p = 4; p <= smax; p *= 2) {
+        tss.push_back((int)p);
+        if (p * 3 / 2 <= smax && p >= 4) tss.push_back((int)(p * 3 / 2));
+    }
+    std::sort(tss.begin(), tss.end());
+    tss.erase(std::unique(tss.begin(), tss.end()), tss.end());
+    std::vector<std::pair<stencil_tile, double>> vals;
+    double bt = std::numeric_limits<double>::infinity();
+    stencil_tile bb{0, 0, 0, 0};
+    for (int t = 1; t <= std::min<int64_t>(T, 128); ++t)
+        for (int ts : tss) {
+            stencil_tile tl{t, ts, 0, 0};
+            const double v = model_predict_wavefront(kind, 1, dims, T, tl, hw);
+            if (!std::isfinite(v)) continue;
+            vals.push_back({tl, v});
+            if (v < bt) { bt = v; bb = tl; }
+        }
+    if (!std::isfinite(bt)) return STENCIL_ETILE;
+    *best = bb;
+    int n = 0;
+    for (auto& e : vals)
+        if (e.second <= (1.0 + within) * bt) {
+            if (cands && n < cap) cands[n] = e.first;
+            ++n;
+        }
+    if (n_cands) *n_cands = n;
+    return STENCIL_OK;
+}
+
 extern "C" int model_select_tile(stencil_kind kind, int ndims, const int64_t* dims, int64_t T,
                                  const model_hw_params* hw, double within, stencil_tile* best, int* best_threads,
                                  stencil_tile* cands, int cap, int* n_cands) {

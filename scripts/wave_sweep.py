@@ -98,6 +98,12 @@ def main():
     res = {"workload": f"W1: Jacobi-1D 3-point fp32, {n - 2} interior points, T={T}, wavefront schedule",
            "n": n, "T": T, "points": pts}
     summarise(res)
+    # Eq. 31 over the whole search space (reading W3): the selected tile measured, gap to the best swept
+    for key, hw in (("select_paper", hwp), ("select_exact", hwe)):
+        sel, cands = hhc.model_select_wavefront_tile((n,), T, hw, 0.10)
+        t = timed(lambda s: hhc.stencil_run_wavefront(h, d_in, d_out, T, sel, s))
+        res[key] = {"tile": list(sel), "texec": t, "gups": (n - 2) * T / t / 1e9,
+                    "gap_vs_best_swept": t / res["best"]["texec"] - 1, "n_candidates_10pct": len(cands)}
     # the hexagonal schedule on the same workload (K0), a few tiles, best kept
     hexpts = []
     for tile in ((64, 2048), (128, 2048), (256, 2048), (128, 4064), (256, 4064)):
@@ -108,7 +114,8 @@ def main():
     os.makedirs(os.path.dirname(args.out), exist_ok=True)
     with open(args.out, "w") as f:
         json.dump(res, f, indent=1)
-    print(json.dumps({k: res[k] for k in ("best", "talg_paper", "talg_exact", "hex_best")}))
+    print(json.dumps({k: res.get(k) for k in ("best", "talg_paper", "talg_exact", "select_paper", "select_exact",
+                                                "hex_best")}))
 
 
 if __name__ == "__main__":

@@ -120,3 +120,17 @@ def test_library_model_matches_oracle(lib, geometry):
     assert n > 60
     assert math.isnan(hhc.model_predict_wavefront((2,), 5, (2, 4), c))
     assert math.isnan(hhc.model_predict_wavefront((100,), 5, (2, 1), c))
+
+
+@pytest.mark.parametrize("geometry", [hhc.PAPER, hhc.EXACT])
+def test_library_select_matches_oracle(lib, geometry):
+    o = mo.gtx980(1, geometry)
+    o.nSM, o.MSM, o.Mblock = 148, 228 * 1024, 227 * 1024
+    c = hhc.make_hw(n_sm=o.nSM, n_v=o.nV, mtb_sm=o.MTBSM, r_sm=o.RSM, m_sm_bytes=o.MSM,
+                    m_block_bytes=o.Mblock, L_s_per_word=o.L, tau_sync_s=o.tau_sync, T_sync_s=o.T_sync,
+                    C_iter_s=o.C_iter, geometry=geometry)
+    for S, T in ((500, 24), (61, 9)):
+        best, cands = hhc.model_select_wavefront_tile((S + 2,), T, c, 0.10)
+        ob, ot, oc = mo.select_tile_wavefront(S, T, o, 0.10)
+        assert best == ob and cands == oc
+        assert ot == min(mo.talg_wavefront_1d(S, T, tl, o) for tl in oc)
