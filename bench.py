@@ -29,7 +29,7 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 CONFIGS = {
-    "C1": dict(kind=1, dims=(256, 256), T=64, tile=(8, 2, 512, 0), threads=256,
+    "C1": dict(kind=1, dims=(256, 256), T=64, tile=(12, 1, 512, 0), threads=384,
                desc="Jacobi-2D 5-point fp32, 256x256, T=64"),
     "C2": dict(kind=2, dims=(8192, 8192), T=1024, tile=(32, 12, 512, 0), threads=384,
                desc="Heat-2D 9-point fp32, 8192x8192, T=1024"),
