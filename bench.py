@@ -3,17 +3,19 @@
 
 A "step" is one pass of the whole hot path (plan, buffer
 setup, every row of hexagons) over one synthetic input: T time steps of the
-config's stencil on its full grid.  N = 1 workload: BASELINE.json configs[1],
-Heat-2D 9-point fp32, 8192^2, T = 1024 (C2).  The tile is the one listed in
-CONFIGS (chosen with model_select_tile + the measured sweep).
+config's stencil on its full grid.  Default workload: C3, Gradient-2D fp32,
+16384^2, T = 512 -- the BASELINE.json config quoted at 1/2/4/8 GPUs, so the
+N = 1 line and the scaling run measure the same problem.  --config C1..C5
+(and the extension configs X1, W1) select the others.  The tile is the one
+listed in CONFIGS (model_select_tile + the measured sweep).
 
-    python bench.py [--gpus N] [--steps K] [--warmup W] [--config C2] [--impl reference]
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config C3] [--impl reference]
 
-Under torchrun (N > 1) the grid is slab-decomposed along S1 across the ranks
-with a ghost exchange (NCCL P2P) every time tile; by default every rank owns a
-config-sized slab (weak scaling: global grid N*(S1-2)+2 rows), --strong splits
-the config's own grid.  Rank 0 prints the line; times are the max over ranks of
-device (CUDA-event) time.
+Under torchrun (N > 1) the config's grid is slab-decomposed along S1 across
+the ranks (strong scaling, the BASELINE 1/2/4/8 experiment) with a ghost
+exchange every time tile; --weak gives every rank a config-sized slab instead.
+Rank 0 prints the line; times are the max over ranks of device (CUDA-event)
+time.
 """
 from __future__ import annotations
 
@@ -46,12 +48,15 @@ CONFIGS = {
     "W1": dict(kind=7, dims=((1 << 22) + 2,), T=1024, tile=(4, 8192), threads=256, schedule="wavefront",
                desc="Jacobi-1D 3-point fp32, 2^22 interior points, T=1024, wavefront schedule (extension f3)"),
 }
-DEFAULT_CONFIG = "C2"
+DEFAULT_CONFIG = "C3"
 
-# Algorithmic FP32 flops per update of the canonical fused expression
-# (DESIGN.md §Roofline): linear kinds 1 mul + (|N|-1) fma = 2|N|-1; Gradient
-# 19 (sqrt and div counted as one flop each, their SASS sequences are longer).
-FLOPS_PER_UPDATE = {1: 9, 2: 17, 3: 19, 4: 13, 5: 53, 6: 9, 7: 5}
+# n_fp32 of SURVEY §8(d): FP32-pipe instructions per update (one FFMA/FMUL/FADD
+# lane operation each; a packed FFMA2 counts 2).  Linear kinds: |N| (1 FMUL +
+# |N|-1 FFMA of the canonical fused expression).  Gradient-2D: counted in the
+# kernel's SASS (FP32-pipe lane ops of the IEEE sqrt and division sequences
+# included, MUFU excluded), scripts/count_fp32.py -> profiles/r02/n_fp32_gradient.txt.
+N_FP32 = {1: 5, 2: 9, 3: 25, 4: 7, 5: 27, 6: 5, 7: 3}
+N_FP32_SOURCE = {3: "SASS count of the Gradient-2D row step (profiles/r02/n_fp32_gradient.txt)"}
 
 METRIC = "GStencil-updates/s"
 
@@ -65,10 +70,27 @@ def load_peaks():
         return {}
 
 
-def fp32_peak_tflops(peaks) -> float:
-    """FP32 FMA peak: 148 SMs x 128 lanes x 2 flops x max SM clock."""
+def p_fma(peaks) -> float:
+    """P_fma of SURVEY §8(d): FP32-pipe lane instructions per second = 148 SMs x
+    128 FP32 lanes x max SM clock (MEASURED_PEAKS.json sm_max_mhz); measured on
+    this B200 at 120-126 FMA/clk/SM (scripts/ubench/ffma2.cu, profiles/r02/probe)."""
     mhz = float(peaks.get("sm_max_mhz", 1965.0))
-    return 148 * 128 * 2 * mhz * 1e6 / 1e12
+    return 148 * 128 * mhz * 1e6
+
+
+def alu_roofline(kind: int, upd_per_s: float, peaks: dict, **extra) -> dict:
+    """roofline = P_fma / n_fp32 updates/s; frac = achieved / that."""
+    n = N_FP32[kind]
+    peak = p_fma(peaks) / n / 1e9
+    ach = upd_per_s / 1e9
+    d = {"bound": "alu", "achieved": round(ach, 3), "peak": round(peak, 2), "unit": "GStencil-updates/s",
+         "frac": round(ach / peak, 4), "n_fp32": n,
+         "peak_basis": "P_fma / n_fp32: 148 SM x 128 FP32 lanes x sm_max_mhz (MEASURED_PEAKS.json) "
+                       "FP32-pipe instr/s over n_fp32 per update (SURVEY 8(d))"}
+    if kind in N_FP32_SOURCE:
+        d["n_fp32_source"] = N_FP32_SOURCE[kind]
+    d.update(extra)
+    return d
 
 
 class ClockSampler:
@@ -206,9 +228,9 @@ def main(argv=None):
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-overlap", action="store_true",
                     help="N>1: exchange, then the whole ghost-extended slab (no overlap)")
-    ap.add_argument("--strong", action="store_true",
-                    help="N > 1: split the config's grid over the ranks (default: weak scaling, one config-sized "
-                         "slab per rank)")
+    ap.add_argument("--weak", action="store_true",
+                    help="N > 1: one config-sized slab per rank (default: strong scaling, the config's grid split "
+                         "over the ranks)")
     args = ap.parse_args(argv)
     cfg = CONFIGS[args.config]
     if args.impl == "reference":
@@ -279,17 +301,13 @@ def bench_single(args, cfg, cfgname):
         ksec, klaunch = dt / args.steps, launches_per_step - 2
     else:
         ksec, klaunch = hhc.stencil_profile(s, d_in, d_out, T, tile, threads, stream)
-    flops = FLOPS_PER_UPDATE[kind] * n_upd
-    peaks = load_peaks()
-    peak = fp32_peak_tflops(peaks)
-    achieved = flops / ksec / 1e12
     traffic = ncu_traffic(cfgname)
-    roofline = {"bound": "alu", "achieved": round(achieved, 3), "peak": round(peak, 2), "unit": "TFLOP/s",
-                "frac": round(achieved / peak, 4), "traffic": traffic,
-                "kernel": "wave1d_kernel" if wave else {1: "hex1d_kernel", 2: "hex2d_kernel", 3: "hex3d_kernel"}[len(dims)],
-                "kernel_share_of_step": round(ksec / (dt / args.steps), 4),
-                "kernel_launches_per_step": klaunch,
-                "peak_basis": "148 SM x 128 FP32 lanes x 2 x sm_max_mhz (MEASURED_PEAKS.json)"}
+    roofline = alu_roofline(kind, n_upd / ksec, load_peaks(), traffic=traffic,
+                            kernel="wave1d_kernel" if wave else {1: "hex1d_kernel", 2: "hex2d_kernel",
+                                                                 3: "hex3d_kernel"}[len(dims)],
+                            kernel_share_of_step=round(ksec / (dt / args.steps), 4),
+                            kernel_launches_per_step=klaunch,
+                            achieved_basis="updates per step / summed CUDA-event time of the HHC row launches")
 
     e2e = None
     if not args.no_e2e:

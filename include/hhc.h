@@ -88,6 +88,8 @@ typedef struct {
     int32_t n_gpus;            /* >1: slab decomposition model (M7)           */
     double  link_bytes_per_s;  /* per-direction GPU-GPU bandwidth                       */
     double  link_latency_s;    /* per-message latency                                   */
+    int32_t dist_overlap;      /* M7: 0 = exchange then the ghost-extended slab, 1 =
+                                  edge sub-slabs overlapped with the interior           */
 } model_hw_params;
 
 typedef struct stencil_s* stencil_t;     /* opaque; owned by the library */
@@ -141,10 +143,21 @@ int model_select_tile(stencil_kind kind, int ndims, const int64_t* dims, int64_t
                       stencil_tile* best, int* best_threads,
                       stencil_tile* cands, int cap, int* n_cands);
 
-/* Shared-memory bytes and threads the kernel uses for (ndims, tile, threads);
- * 0 / error if the tile is invalid.  Lets callers and the model agree on Mtile. */
-int stencil_tile_resources(int ndims, stencil_tile tile, int threads,
+/* Resources of the HHC kernel the library launches for (kind, ndims, tile,
+ * threads, mode) with default weights: shared-memory bytes per block (Mtile,
+ * Eq. 19 / reading M3), threads per block, and registers per thread from
+ * cudaFuncGetAttributes -- the Rtile of Eq. 11 the paper could not know
+ * (reading M4).  *regs_per_thread = 0 when kind = 0 or
+ * no CUDA device is visible.  STENCIL_ETILE / STENCIL_EINVAL if the tile or
+ * threads are invalid (then nothing is written).  Host only; no allocation. */
+int stencil_tile_resources(stencil_kind kind, int ndims, stencil_tile tile, int threads, int mode,
                            int64_t* smem_bytes, int* block_threads, int* regs_per_thread);
+
+/* Resident blocks per SM of that kernel (cudaOccupancyMaxActiveBlocksPerMultiprocessor
+ * at its dynamic shared memory): the k of Eq. 11 as the hardware sees it,
+ * against which the EXACT model's k is tested.  Needs a device (STENCIL_ENODEV). */
+int stencil_tile_occupancy(stencil_kind kind, int ndims, stencil_tile tile, int threads, int mode,
+                           int* blocks_per_sm);
 
 /* Launch geometry of a run: number of hexagon rows (kernel launches, Nw) and
  * the number of thread blocks of phase-A and phase-B rows (w(i), Eq. 5). */

@@ -54,7 +54,7 @@ class model_hw_params(ctypes.Structure):
                 ("regs_per_thread", ctypes.c_int32), ("geometry", ctypes.c_int32),
                 ("threads", ctypes.c_int32), ("max_threads_sm", ctypes.c_int32),
                 ("n_gpus", ctypes.c_int32), ("link_bytes_per_s", ctypes.c_double),
-                ("link_latency_s", ctypes.c_double)]
+                ("link_latency_s", ctypes.c_double), ("dist_overlap", ctypes.c_int32)]
 
 
 def make_tile(t) -> stencil_tile:
@@ -104,7 +104,9 @@ def load(build_if_missing: bool = False):
     lib.model_select_tile.argtypes = [ctypes.c_int, ctypes.c_int, i64p, ctypes.c_int64, P(model_hw_params),
                                       ctypes.c_double, P(stencil_tile), P(ctypes.c_int), P(stencil_tile),
                                       ctypes.c_int, P(ctypes.c_int)]
-    lib.stencil_tile_resources.argtypes = [ctypes.c_int, stencil_tile, ctypes.c_int, i64p, P(ctypes.c_int),
+    lib.stencil_tile_resources.argtypes = [ctypes.c_int, ctypes.c_int, stencil_tile, ctypes.c_int, ctypes.c_int,
+                                           i64p, P(ctypes.c_int), P(ctypes.c_int)]
+    lib.stencil_tile_occupancy.argtypes = [ctypes.c_int, ctypes.c_int, stencil_tile, ctypes.c_int, ctypes.c_int,
                                            P(ctypes.c_int)]
     lib.stencil_plan_info.argtypes = [ctypes.c_int, i64p, ctypes.c_int64, stencil_tile, i64p, i64p, i64p, i64p]
     lib.stencil_microbench.argtypes = [ctypes.c_int, ctypes.c_int, ctypes.c_int, i64p, ctypes.c_int64,
@@ -278,13 +280,24 @@ def model_select_tile(kind: int, dims, T: int, hw: model_hw_params, within: floa
     return best.astuple(), thr.value, [cands[i].astuple() for i in range(min(n.value, cap))]
 
 
-def stencil_tile_resources(ndims: int, tile, threads: int = 0):
+def stencil_tile_resources(ndims: int, tile, threads: int = 0, kind: int = 0, mode: int = FUSED):
+    """(smem bytes, threads per block, registers per thread) of the kernel the
+    library launches; registers are 0 for kind = 0 or without a CUDA device."""
     sm = ctypes.c_int64()
     thr = ctypes.c_int()
     regs = ctypes.c_int()
-    _check(load().stencil_tile_resources(int(ndims), make_tile(tile), int(threads), ctypes.byref(sm),
-                                         ctypes.byref(thr), ctypes.byref(regs)), "stencil_tile_resources")
-    return sm.value, thr.value
+    _check(load().stencil_tile_resources(int(kind), int(ndims), make_tile(tile), int(threads), int(mode),
+                                         ctypes.byref(sm), ctypes.byref(thr), ctypes.byref(regs)),
+           "stencil_tile_resources")
+    return sm.value, thr.value, regs.value
+
+
+def stencil_tile_occupancy(kind: int, tile, threads: int = 0, mode: int = FUSED) -> int:
+    """Resident blocks per SM of the kernel for (kind, tile, threads) (CUDA occupancy API)."""
+    k = ctypes.c_int()
+    _check(load().stencil_tile_occupancy(int(kind), KIND_NDIMS[int(kind)], make_tile(tile), int(threads), int(mode),
+                                         ctypes.byref(k)), "stencil_tile_occupancy")
+    return k.value
 
 
 def stencil_plan_info(dims, T: int, tile):
@@ -310,7 +323,7 @@ def updates(dims, T: int) -> int:
 
 
 EXPORTED_SYMBOLS = ["stencil_create", "stencil_destroy", "stencil_run", "stencil_run_host",
-                    "stencil_run_planes", "model_predict", "model_select_tile", "stencil_tile_resources",
+                    "stencil_run_planes", "model_predict", "model_select_tile", "stencil_tile_resources", "stencil_tile_occupancy",
                     "stencil_plan_info", "stencil_microbench", "stencil_strerror", "stencil_last_launches",
                     "stencil_profile", "stencil_run_wavefront", "stencil_wavefront_info",
                     "model_predict_wavefront", "model_select_wavefront_tile"]

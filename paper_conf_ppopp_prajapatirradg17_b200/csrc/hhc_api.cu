@@ -64,7 +64,6 @@ struct RunSpec {
     int64_t T;
     stencil_tile tile;
     int G, thr;
-    int nr;                   // > 0: register-resident 2D kernel K1R with NR rows
 };
 
 struct GraphEntry {
@@ -95,6 +94,7 @@ struct stencil_s {
     uint64_t use_clock = 0;
     int compute_only = 0;
     int occ = 1;
+    int envJ = 0;               // HHC_J read once at create (experiments; 0 = library rule)
 
     int64_t nelem() const { return dims[0] * dims[1] * dims[2]; }
 };
@@ -110,6 +110,11 @@ extern "C" const char* stencil_strerror(int status) {
     case STENCIL_ENODEV: return "no usable sm_100 device";
     default: return "unknown status";
     }
+}
+
+static void drop_graphs(stencil_t h) {
+    for (auto& g : h->graphs) cudaGraphExecDestroy(g.exec);
+    h->graphs.clear();
 }
 
 static int cuda_fail(stencil_t h, cudaError_t e) {
@@ -164,6 +169,7 @@ extern "C" int stencil_create(stencil_kind kind, int ndims, const int64_t* dims,
             if (ncoeffs == n + 1 && coeffs[n] != 0.0f) { h->has_c = true; h->c = coeffs[n]; h->defw = false; }
         }
     }
+    if (const char* ej = getenv("HHC_J")) h->envJ = std::max(0, atoi(ej));
     if (cudaStreamCreateWithFlags(&h->cap_stream, cudaStreamNonBlocking) != cudaSuccess) {
         delete h;
         return STENCIL_ECUDA;
@@ -174,7 +180,7 @@ extern "C" int stencil_create(stencil_kind kind, int ndims, const int64_t* dims,
 
 extern "C" void stencil_destroy(stencil_t h) {
     if (!h) return;
-    for (auto& g : h->graphs) cudaGraphExecDestroy(g.exec);
+    drop_graphs(h);
     if (h->scratch) cudaFree(h->scratch);
     if (h->flags) cudaFree(h->flags);
     if (h->h_in_dev) cudaFree(h->h_in_dev);
@@ -217,15 +223,40 @@ static int check_tile(int ndims, stencil_tile t, int threads, int smem_limit, in
     return STENCIL_OK;
 }
 
-extern "C" int stencil_tile_resources(int ndims, stencil_tile tile, int threads, int64_t* smem,
-                                      int* block_threads, int* regs) {
+extern "C" int stencil_tile_resources(stencil_kind kind, int ndims, stencil_tile tile, int threads, int mode,
+                                      int64_t* smem, int* block_threads, int* regs) {
     if (ndims < 1 || ndims > 3) return STENCIL_EINVAL;
+    if (kind != 0 && kind_ndims_host(kind) != ndims) return STENCIL_EINVAL;
     int G, thr;
     const int rc = check_tile(ndims, tile, threads, 227 * 1024, &G, &thr);
     if (rc) return rc;
     if (smem) *smem = smem_bytes(ndims, tile.t, tile.s1, tile.s2, tile.s3);
     if (block_threads) *block_threads = thr;
-    if (regs) *regs = 0;
+    if (regs) {
+        // Eq. 11's register bound (reading M4): the kernel the library launches for this
+        // (kind, mode, tile) with default weights, from cudaFuncGetAttributes; 0 if kind is 0
+        // or no device is visible (the attribute query needs a CUDA context)
+        *regs = kind != 0 ? hex_kernel_regs(ndims, kind, mode, false, true, tile.s2) : 0;
+        cudaGetLastError();
+    }
+    return STENCIL_OK;
+}
+
+extern "C" int stencil_tile_occupancy(stencil_kind kind, int ndims, stencil_tile tile, int threads, int mode,
+                                      int* blocks_per_sm) {
+    if (!blocks_per_sm || kind_ndims_host(kind) != ndims) return STENCIL_EINVAL;
+    int G, thr;
+    const int rc = check_tile(ndims, tile, threads, 227 * 1024, &G, &thr);
+    if (rc) return rc;
+    hex_kernel_t k = get_hex_kernel(ndims, kind, mode, false, true, tile.s2);
+    if (!k) return STENCIL_EINVAL;
+    const int64_t smem = smem_bytes(ndims, tile.t, tile.s1, tile.s2, tile.s3);
+    cudaError_t e = cudaFuncSetAttribute((const void*)k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, (const void*)k, thr, (size_t)smem);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        return e == cudaErrorNoDevice || e == cudaErrorInsufficientDriver ? STENCIL_ENODEV : STENCIL_ECUDA;
+    }
     return STENCIL_OK;
 }
 
@@ -287,15 +318,13 @@ extern "C" int stencil_plan_info(int ndims, const int64_t* dims, int64_t T, sten
 static int choose_J(stencil_t h, const RowPlan& r) {
     const int cap = std::max(1, h->nsm * std::max(h->occ, 1) / std::max(r.w, 1));
     int J = std::max(1, std::min(r.n2, cap));
-    const char* envJ = getenv("HHC_J");
-    if (envJ) J = std::max(1, std::min({atoi(envJ), r.n2, cap}));
+    if (h->envJ > 0) J = std::max(1, std::min({h->envJ, r.n2, cap}));
     return J;
 }
 
 // Everything that must not happen inside stream capture: the kernel's smem
 // attribute, its occupancy (for J), and the 3D flag buffer.
-static int prepare_rows(stencil_t h, const int64_t* dims, int64_t T, stencil_tile tile, int thr, int nr = 0) {
-    (void)nr;
+static int prepare_rows(stencil_t h, const int64_t* dims, int64_t T, stencil_tile tile, int thr) {
     hex_kernel_t k = get_hex_kernel(h->ndims, h->kind, h->mode, h->has_c, h->defw, tile.s2);
     if (!k) return STENCIL_EINVAL;
     const int64_t smem = smem_bytes(h->ndims, tile.t, tile.s1, tile.s2, tile.s3);
@@ -314,6 +343,9 @@ static int prepare_rows(stencil_t h, const int64_t* dims, int64_t T, stencil_til
         if (J > 1) need = std::max<int64_t>(need, (int64_t)r.w * r.n2);
     }
     if (need > h->flags_n) {
+        // the cached graphs captured the old flag pointer (memset node and kernel
+        // parameters): they must not be replayed after the buffer moves
+        drop_graphs(h);
         if (h->flags) cudaFree(h->flags);
         h->flags = nullptr;
         h->flags_n = 0;
@@ -329,10 +361,9 @@ static int prepare_rows(stencil_t h, const int64_t* dims, int64_t T, stencil_til
 // result (level T) lands in plane[T & 1].  Ring values are read from `ring`.
 static int enqueue_rows(stencil_t h, const int64_t* dims, const float* ring, float* plane0, float* plane1,
                         int64_t T, stencil_tile tile, int G, int thr, cudaStream_t s, int64_t* launches,
-                        std::vector<cudaEvent_t>* evs = nullptr, int nr = 0) {
+                        std::vector<cudaEvent_t>* evs = nullptr) {
     std::vector<RowPlan> rows;
     plan_rows(h->ndims, dims, T, tile, rows);
-    (void)nr;
     hex_kernel_t k = get_hex_kernel(h->ndims, h->kind, h->mode, h->has_c, h->defw, tile.s2);
     if (!k) return STENCIL_EINVAL;
     const int64_t smem = smem_bytes(h->ndims, tile.t, tile.s1, tile.s2, tile.s3);
@@ -368,7 +399,6 @@ static int enqueue_rows(stencil_t h, const int64_t* dims, const float* ring, flo
     p.kappa = h->kappa;
     p.flags = h->flags;
     p.compute_only = h->compute_only;
-    { static const int dbg = getenv("HHC_DBG") ? atoi(getenv("HHC_DBG")) : 0; p.dbg = dbg; }
     for (auto& r : rows) {
         p.t0 = r.t0; p.xbase = r.xbase; p.tau_lo = r.tau_lo; p.tau_hi = r.tau_hi;
         p.n2 = r.n2; p.n3 = r.n3; p.J = r.J;
@@ -405,11 +435,11 @@ static int enqueue_spec(stencil_t h, const RunSpec& r, cudaStream_t s, int64_t* 
         // a2: level 0 in plane 0, the fixed ring in plane 1 (readings R2/R3)
         launch_copy_full(r.a, plane[0], n, s); ++nl;
         launch_copy_ring(r.a, plane[1], r.dims[0], r.dims[1], r.dims[2], s); ++nl;
-        rc = enqueue_rows(h, r.dims, r.a, plane[0], plane[1], r.T, r.tile, r.G, r.thr, s, &nrows, nullptr, r.nr);
+        rc = enqueue_rows(h, r.dims, r.a, plane[0], plane[1], r.T, r.tile, r.G, r.thr, s, &nrows, nullptr);
     } else {
         float* p0 = const_cast<float*>(r.a);
         launch_copy_ring(p0, r.b, r.dims[0], r.dims[1], r.dims[2], s); ++nl;
-        rc = enqueue_rows(h, r.dims, p0, p0, r.b, r.T, r.tile, r.G, r.thr, s, &nrows, nullptr, r.nr);
+        rc = enqueue_rows(h, r.dims, p0, p0, r.b, r.T, r.tile, r.G, r.thr, s, &nrows, nullptr);
     }
     *launches = nl + nrows;
     return rc;
@@ -419,12 +449,12 @@ static bool same_spec(const RunSpec& x, const RunSpec& y) {
     return x.planes_mode == y.planes_mode && x.a == y.a && x.b == y.b && x.dims[0] == y.dims[0] &&
            x.dims[1] == y.dims[1] && x.dims[2] == y.dims[2] && x.T == y.T && x.tile.t == y.tile.t &&
            x.tile.s1 == y.tile.s1 && x.tile.s2 == y.tile.s2 && x.tile.s3 == y.tile.s3 && x.G == y.G &&
-           x.thr == y.thr && x.nr == y.nr;
+           x.thr == y.thr;
 }
 
 // Run a spec through the CUDA-graph cache (captured once per spec, replayed).
 static int run_spec(stencil_t h, const RunSpec& r, cudaStream_t s) {
-    int prc = r.planes_mode == 2 ? STENCIL_OK : prepare_rows(h, r.dims, r.T, r.tile, r.thr, r.nr);
+    int prc = r.planes_mode == 2 ? STENCIL_OK : prepare_rows(h, r.dims, r.T, r.tile, r.thr);
     if (prc) return prc;
     const bool use_graph = getenv("HHC_NO_GRAPH") == nullptr && !h->compute_only;
     if (!use_graph) {
@@ -487,7 +517,6 @@ extern "C" int stencil_run(stencil_t h, const float* d_in, float* d_out, int64_t
         if (e != cudaSuccess) { h->scratch = nullptr; return STENCIL_ENOMEM; }
     }
     r.planes_mode = 0; r.a = d_in; r.b = d_out;
-    r.nr = 0;
     for (int d = 0; d < 3; ++d) r.dims[d] = h->dims[d];
     r.T = T; r.tile = tile;
     if (h->ndims == 2) r.tile.s3 = 0;
@@ -504,7 +533,6 @@ extern "C" int stencil_run_planes(stencil_t h, int64_t rows, float* plane0, floa
     if (rc) return rc;
     cudaSetDevice(h->device);
     r.planes_mode = 1; r.a = plane0; r.b = plane1;
-    r.nr = 0;
     r.dims[0] = rows; r.dims[1] = h->dims[1]; r.dims[2] = h->dims[2];
     const int64_t n = r.dims[0] * r.dims[1] * r.dims[2];
     if (plane1 < plane0 + n && plane0 < plane1 + n) return STENCIL_EINVAL;
@@ -605,7 +633,7 @@ extern "C" int stencil_run_wavefront(stencil_t h, const float* d_in, float* d_ou
     r.planes_mode = 2; r.a = d_in; r.b = d_out;
     r.dims[0] = n; r.dims[1] = 1; r.dims[2] = 1;
     r.T = T; r.tile = tile; r.tile.s2 = r.tile.s3 = 0;
-    r.G = 1; r.thr = 256; r.nr = 0;
+    r.G = 1; r.thr = 256;
     return run_spec(h, r, s);
 }
 
@@ -630,12 +658,11 @@ extern "C" int stencil_profile(stencil_t h, const float* d_in, float* d_out, int
     plane[1 - (T & 1)] = h->scratch;
     launch_copy_full(d_in, plane[0], n, s);
     launch_copy_ring(d_in, plane[1], h->dims[0], h->dims[1], h->dims[2], s);
-    const int nr = 0;
-    rc = prepare_rows(h, h->dims, T, tile, thr, nr);
+    rc = prepare_rows(h, h->dims, T, tile, thr);
     if (rc) return rc;
     std::vector<cudaEvent_t> evs;
     int64_t nl = 0;
-    rc = enqueue_rows(h, h->dims, d_in, plane[0], plane[1], T, tile, G, thr, s, &nl, &evs, nr);
+    rc = enqueue_rows(h, h->dims, d_in, plane[0], plane[1], T, tile, G, thr, s, &nl, &evs);
     if (rc == STENCIL_OK) rc = cuda_fail(h, cudaStreamSynchronize(s));
     double tot = 0.0;
     for (size_t i = 0; i + 1 < evs.size(); i += 2) {

@@ -1,5 +1,5 @@
 // hhc_device.cuh -- device helpers shared by the HHC kernels (hhc_kernels.cu,
-// hhc_kernels_reg.cu): stencil tables, canonical point updates (reading R4),
+// wave_kernels.cu, microbench.cu): stencil tables, canonical point updates (reading R4),
 // hexagon geometry (readings G1-G3), cp.async, the per-block geometry table.
 #pragma once
 #include <cuda_runtime.h>
@@ -158,13 +158,6 @@ __device__ __forceinline__ float lin3(const float (&r0)[3][6], const float (&r1)
 }
 
 // ----------------------------------------------------------------- helpers
-__device__ __forceinline__ void ld10(const float* base, float (&r)[10]) {
-    const float2 h = *reinterpret_cast<const float2*>(base - 2);
-    const float4 m = *reinterpret_cast<const float4*>(base);
-    const float4 q = *reinterpret_cast<const float4*>(base + 4);
-    r[0] = h.x; r[1] = h.y; r[2] = m.x; r[3] = m.y; r[4] = m.z; r[5] = m.w;
-    r[6] = q.x; r[7] = q.y; r[8] = q.z; r[9] = q.w;
-}
 __device__ __forceinline__ void ld6(const float* base, float (&r)[6]) {
     const float2 h = *reinterpret_cast<const float2*>(base - 2);
     const float4 m = *reinterpret_cast<const float4*>(base);
@@ -257,8 +250,7 @@ __device__ __forceinline__ void facet_gap(int64_t nl, int64_t nr, int64_t S1, bo
 // Per-level geometry of the block's hexagon, in smem rows pp = x - xs, computed
 // once per block (identical for every sub-tile); kGeo ints per level:
 //  0..5 footprint intervals f1, f2, inner; 6 first; 7 empty;
-//  8, 9 the row [rl, rr); 10, 11 the non-facet gap [lo, hi); 12 rows per x-group;
-//  13, 14 the bit mask of the footprint rows (register kernel).
+//  8, 9 the row [rl, rr); 10, 11 the non-facet gap [lo, hi); 12 rows per x-group.
 constexpr int kGeo = 16;
 __device__ __forceinline__ void build_geo(const HexParams& p, int64_t x0, int64_t xs, int nlev, int* geo) {
     const int NX = p.tS1 + p.tT + 2;
@@ -278,15 +270,6 @@ __device__ __forceinline__ void build_geo(const HexParams& p, int64_t x0, int64_
         facet_gap(nl, nr, p.S1, tb + lev == p.T, xs, NX, lo, hi);
         g[10] = lo; g[11] = hi;
         g[12] = (int)((rr - rl + p.G - 1) / p.G);
-        // 64-bit mask of the footprint rows F(lev) (register kernel, rows < 64)
-        unsigned long long fm = 0;
-        for (int seg = 0; seg < 2; ++seg)
-            for (int pp = g[2 * seg]; pp < g[2 * seg + 1]; ++pp) {
-                const int64_t x = xs + pp;
-                if (pp >= 0 && pp < 64 && x != 0 && x != p.S1 - 1) fm |= 1ull << pp;   // ring rows excluded
-            }
-        g[13] = (int)(unsigned)(fm & 0xffffffffu);
-        g[14] = (int)(unsigned)(fm >> 32);
     }
 }
 

@@ -32,7 +32,6 @@ struct HexParams {
     float c;                // Eq. 1 constant
     float kappa;            // Gradient-2D
     int compute_only;       // K4: skip all global<->shared transfers (Citer micro-benchmark)
-    int dbg;                // experiment switches (HHC_DBG, never set in production runs)
 };
 
 // Shared-memory bytes of the HHC kernels (DESIGN.md §Kernels K1/K2): two parity

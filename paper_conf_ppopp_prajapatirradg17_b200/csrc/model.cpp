@@ -100,15 +100,26 @@ int default_threads(int nd, const stencil_tile& t) {
     return base * G;
 }
 
+// Eq. 11's k under the CUDA occupancy rules (reading M4): shared memory per block
+// plus the 1 KB the driver reserves per block, registers allocated per warp in
+// units of 256, at most MTBSM blocks and max_threads_sm threads per SM.
+int64_t k_exact(int64_t Mtile, int64_t threads, const model_hw_params& hw) {
+    const int64_t maxthr = hw.max_threads_sm > 0 ? hw.max_threads_sm : 2048;
+    int64_t k = std::min<int64_t>({hw.m_sm_bytes / (Mtile + 1024), (int64_t)hw.mtb_sm, maxthr / threads});
+    if (hw.regs_per_thread > 0) {
+        const int64_t per_warp = cdiv(32 * (int64_t)hw.regs_per_thread, 256) * 256;
+        k = std::min<int64_t>(k, (hw.r_sm / per_warp) / cdiv(threads, 32));
+    }
+    return k;
+}
+
 double talg_exact(int nd, const int64_t* S, int64_t T, const stencil_tile& tl, const model_hw_params& hw) {
     const int64_t tT = tl.t, tS1 = tl.s1, tS2 = tl.s2, tS3 = nd == 3 ? tl.s3 : 1;
     const int64_t S1 = S[0], S2 = S[1], S3 = nd == 3 ? S[2] : 1;
     const int64_t Mtile = hhc::smem_bytes(nd, (int)tT, (int)tS1, (int)tS2, (int)tS3);
     const int threads = hw.threads > 0 ? hw.threads : default_threads(nd, tl);
-    const int64_t maxthr = hw.max_threads_sm > 0 ? hw.max_threads_sm : 2048;
     if (Mtile > hw.m_block_bytes || threads > hhc::max_block_threads(nd)) return std::numeric_limits<double>::infinity();
-    int64_t k = std::min<int64_t>({hw.m_sm_bytes / Mtile, (int64_t)hw.mtb_sm, maxthr / threads});   // Eq. 11
-    if (hw.regs_per_thread > 0) k = std::min<int64_t>(k, hw.r_sm / ((int64_t)hw.regs_per_thread * threads));
+    const int64_t k = k_exact(Mtile, threads, hw);                                       // Eq. 11
     if (k < 1) return std::numeric_limits<double>::infinity();
     const int64_t P = 2 * tS1 + tT, h = tT / 2;
     const int64_t wA = cdiv(S1 + h, P);                        // reading G2
@@ -177,22 +188,46 @@ double talg_exact(int nd, const int64_t* S, int64_t T, const stencil_tile& tl, c
     return total;
 }
 
-// Reading M7 (multi-GPU, not in the paper): G slabs of own = ceil(S1/G) rows,
-// each time tile of tT steps runs HHC on own + 2 tT rows and exchanges tT rows
-// per neighbour: T_G = ceil(T/tT) * (Talg(own + 2 tT, tT) + T_exch).
+// Reading M7 (multi-GPU, not in the paper; BASELINE.json north_star): G slabs of
+// own = ceil(S1/G) interior rows along S1, ghost depth g = tT, time tiles of
+// Tt = tT steps (the last one T - (n-1) tT).  The busiest rank has e = 2
+// neighbours (e = 1 when G = 2).  Per tile, with T_exch = g * plane * 4 B / link
+// bandwidth + latency:
+//   plain   (dist_overlap = 0): Talg(own + e g, Tt) + T_exch
+//   overlap (dist_overlap = 1): Talg(own, Tt) + e Talg(3 g, Tt) + max(0, T_exch - Talg(own, Tt))
+// (the edge sub-slabs of 3g rows run besides the ghost-free interior, which hides
+// the exchange).  T_G = the sum over the tiles.
 double talg_dist(int nd, const int64_t* S, int64_t T, const stencil_tile& tl, const model_hw_params& hw,
                  double (*f)(int, const int64_t*, int64_t, const stencil_tile&, const model_hw_params&)) {
     const int64_t G = hw.n_gpus;
+    const int64_t g = tl.t;
     const int64_t own = cdiv(S[0], G);
-    int64_t Sl[3] = {own + 2 * tl.t, S[1], nd == 3 ? S[2] : 1};
-    const int64_t ntile = cdiv(T, tl.t);
-    double tile_time = f(nd, Sl, tl.t, tl, hw);
-    if (!std::isfinite(tile_time)) return tile_time;
+    const int64_t e = G >= 3 ? 2 : 1;
     const double plane = (double)S[1] * (double)(nd == 3 ? S[2] : 1) * 4.0;
-    const double msg = (double)tl.t * plane;
     const double bw = hw.link_bytes_per_s > 0 ? hw.link_bytes_per_s : 7.7e11;
-    const double t_exch = msg / bw + hw.link_latency_s;
-    return (double)ntile * (tile_time + t_exch);
+    const double t_exch = (double)g * plane / bw + hw.link_latency_s;
+    auto run = [&](int64_t rows, int64_t Tt) {
+        const int64_t Sl[3] = {rows, S[1], nd == 3 ? S[2] : 1};
+        return f(nd, Sl, Tt, tl, hw);
+    };
+    const int64_t n = cdiv(T, tl.t);
+    const int64_t Tlast = T - (n - 1) * tl.t;
+    double total = 0.0;
+    for (int pass = 0; pass < 2; ++pass) {            // pass 0: the n-1 full tiles, pass 1: the last one
+        const int64_t Tt = pass == 0 ? tl.t : Tlast;
+        const int64_t cnt = pass == 0 ? n - 1 : 1;
+        if (cnt == 0) continue;
+        double tt;
+        if (hw.dist_overlap && own >= 2 * g) {
+            const double ti = run(own, Tt);
+            tt = ti + (double)e * run(3 * g, Tt) + std::max(0.0, t_exch - ti);
+        } else {
+            tt = run(own + e * g, Tt) + t_exch;
+        }
+        if (!std::isfinite(tt)) return tt;
+        total += (double)cnt * tt;
+    }
+    return total;
 }
 
 }  // namespace
@@ -230,10 +265,7 @@ extern "C" double model_predict_wavefront(stencil_kind kind, int ndims, const in
     const int64_t Mtile = hhc::wave1d_smem_bytes(tile.t, tile.s1);
     if (Mtile > hw->m_block_bytes) return inf;
     int64_t k = std::min<int64_t>(hw->m_sm_bytes / Mtile, hw->mtb_sm);         // Eq. 11
-    if (hw->geometry == 1) {
-        k = std::min<int64_t>(k, (hw->max_threads_sm > 0 ? hw->max_threads_sm : 2048) / 256);
-        if (hw->regs_per_thread > 0) k = std::min<int64_t>(k, hw->r_sm / (hw->regs_per_thread * 256));
-    }
+    if (hw->geometry == 1) k = k_exact(Mtile, 256, *hw);                        // reading M4
     if (k < 1) return inf;
     const double L = hw->geometry == 1 ? hw->L_s_per_word * hw->n_sm : hw->L_s_per_word;   // reading M5
     std::vector<hhc::WaveLaunch> ws;

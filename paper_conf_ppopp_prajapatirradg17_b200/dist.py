@@ -232,7 +232,7 @@ def bench_main(args, cfg, cfgname, configs):
     tile = tile + (0,) * (4 - len(tile))
     threads = cfg["threads"] if args.threads is None else args.threads
     dims, T, kind = cfg["dims"], cfg["T"], cfg["kind"]
-    strong = bool(getattr(args, "strong", False))
+    strong = not bool(getattr(args, "weak", False))
     if not strong:
         # weak scaling (default): every rank owns a slab of the config's interior
         # rows, the global grid is world times taller; ghost exchange as usual
@@ -318,9 +318,6 @@ def bench_main(args, cfg, cfgname, configs):
                "h2d_bytes_per_step": int(nb[0].item()), "d2h_bytes_per_step": int(nb[1].item())}
     n_upd = hhc.updates(dims, T)
     if rank == 0:
-        flops = bench.FLOPS_PER_UPDATE[kind] * n_upd * args.steps
-        peak = bench.fp32_peak_tflops(bench.load_peaks())
-        ach = flops / dt / world / 1e12
         line = {"metric": "GStencil-updates/s", "value": round(n_upd * args.steps / dt / 1e9, 3),
                 "unit": "GStencil-updates/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
                 "ms_per_step": round(dt / args.steps * 1e3, 3), "higher_is_better": True, "scaling": "strong" if strong else "weak",
@@ -332,11 +329,12 @@ def bench_main(args, cfg, cfgname, configs):
                                           + (", exchange overlapped with the interior sub-slab (edge sub-slabs "
                                              "first on a second stream)" if overlap else ""),
                            "l2": "inputs larger than L2"},
-                "roofline": {"bound": "alu", "achieved": round(ach, 3), "peak": round(peak, 2), "unit": "TFLOP/s",
-                             "frac": round(ach / peak, 4), "traffic": None,
-                             "kernel": "hex2d_kernel" if len(dims) == 2 else "hex3d_kernel",
-                             "basis": "whole-job algorithmic flops / (max-over-ranks step time x n_gpus), "
-                                      "ghost-row redundancy and exchange included"},
+                "roofline": bench.alu_roofline(kind, n_upd * args.steps / dt / world, bench.load_peaks(),
+                                               traffic=None,
+                                               kernel="hex2d_kernel" if len(dims) == 2 else "hex3d_kernel",
+                                               achieved_basis="updates per GPU per second of the whole step "
+                                                              "(max over ranks; redundancy and exchange "
+                                                              "included)"),
                 "e2e": e2e, "clocks": clocks, "gpu_launches": n_launch}
         print(json.dumps(line))
     hhc.stencil_destroy(h)

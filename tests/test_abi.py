@@ -63,7 +63,8 @@ def test_tile_validation(lib):
         hhc.stencil_tile_resources(2, (64, 64, 1024))
     with pytest.raises(hhc.StencilError):                              # threads not a multiple
         hhc.stencil_tile_resources(2, (8, 8, 64), threads=20)
-    sm, thr = hhc.stencil_tile_resources(3, (8, 4, 4, 32))
+    sm, thr, regs = hhc.stencil_tile_resources(3, (8, 4, 4, 32), kind=hhc.HEAT3D_7PT)
+    assert regs >= 0                                                  # 0 without a device (unknown)
     assert sm == mo.smem_bytes_exact(3, (8, 4, 4, 32)) and thr == mo.default_threads(3, (8, 4, 4, 32))
 
 
@@ -125,6 +126,40 @@ def test_model_predict_matches_oracle_random(lib, geometry):
             n += 1
             assert abs(got - exp) <= 1e-12 * exp, (kind, S, T, tile, got, exp)
     assert n > 100
+
+
+@pytest.mark.parametrize("overlap", [0, 1])
+def test_model_predict_multi_gpu_matches_oracle(lib, overlap):
+    """Reading M7 (the slab model, BASELINE north_star): C++ talg_dist vs the
+    oracle's transcription, random problems, G in 2..8, both exchange variants,
+    both geometries."""
+    rnd = random.Random(70 + overlap)
+    n = 0
+    for _ in range(200):
+        kind = rnd.choice([1, 2, 3, 4, 5])
+        nd = hhc.KIND_NDIMS[kind]
+        geometry = rnd.choice([hhc.PAPER, hhc.EXACT])
+        o, c = hw_pair(kind, geometry, rnd, b200=True)
+        G = rnd.randint(2, 8)
+        o.n_gpus = c.n_gpus = G
+        o.link_Bps = c.link_bytes_per_s = rnd.choice([0.0, 7.7e11, 5e10])
+        o.link_lat = c.link_latency_s = rnd.choice([0.0, 1e-5])
+        o.dist_overlap = c.dist_overlap = overlap
+        if nd == 2:
+            S = (rnd.randint(50, 3000), rnd.randint(1, 2000))
+            tile = (2 * rnd.randint(1, 12), rnd.randint(1, 30), 32 * rnd.randint(1, 8), 0)
+        else:
+            S = (rnd.randint(30, 300), rnd.randint(1, 200), rnd.randint(1, 200))
+            tile = (2 * rnd.randint(1, 6), rnd.randint(1, 10), rnd.randint(1, 8), 32 * rnd.randint(1, 3))
+        T = rnd.randint(1, 300)
+        got = hhc.model_predict(kind, tuple(s + 2 for s in S), T, tile, c)
+        exp = mo.talg(nd, S, T, tile, o)
+        if math.isinf(exp):
+            assert math.isinf(got)
+        else:
+            n += 1
+            assert abs(got - exp) <= 1e-12 * exp, (kind, S, T, tile, G, got, exp)
+    assert n > 50
 
 
 def test_model_predict_invalid_and_infeasible(lib):

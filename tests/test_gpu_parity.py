@@ -2,8 +2,8 @@
 element by element on the same seeded inputs.  Bar (BASELINE.json north_star,
 DESIGN.md R4/R5): bit-exact in both arithmetic modes (plain vs plain oracle,
 fused vs fused oracle); fused within 1e-5 max relative error of the plain
-oracle.  At the full config sizes: exact corner windows (dependence-cone
-argument) plus closed-form / invariant checks over the whole grid."""
+oracle.  The full config sizes in the bench's launch configuration are in
+tests/test_gpu_fullgrid.py."""
 import math
 import os
 
@@ -137,86 +137,6 @@ def test_parity_mid_size(kind, dims, T, tile):
         assert_bits(got, exp, f"{kind} {dims} mode {mode}")
     plain = oracle.run(kind, a, T, hhc.PLAIN)
     assert max_rel(gpu_run(kind, a, T, tile, hhc.FUSED), plain) <= 1e-5
-
-
-# ---- full BASELINE.json sizes, in the launch configuration bench.py times
-FULL = [
-    ("C1", hhc.JACOBI2D_5PT, (256, 256), 64),
-    ("C2", hhc.HEAT2D_9PT, (8192, 8192), 1024),
-    ("C3", hhc.GRADIENT2D, (16384, 16384), 512),
-    ("C4", hhc.HEAT3D_7PT, (512, 512, 512), 256),
-    ("C5", hhc.LAPLACIAN3D_27PT, (768, 768, 768), 128),
-]
-
-
-def bench_tile(cfg):
-    import bench
-    return bench.CONFIGS[cfg]["tile"]
-
-
-@pytest.mark.parametrize("cfg,kind,dims,T", FULL)
-def test_full_size_corner_windows(cfg, kind, dims, T):
-    """Exact check at the full size: out(T, s) depends only on in within
-    distance T of s, so the oracle on a corner window of side T+6 (its far
-    faces act as a fake ring) is exact on the 4-cell corner block."""
-    from synth import CONFIG_SEEDS
-    a = field(CONFIG_SEEDS[cfg], dims)
-    tile = bench_tile(cfg)
-    got = gpu_run(kind, a, T, tile, hhc.FUSED)
-    K = T + 6
-    nd = len(dims)
-    for corner in range(2 ** nd if nd == 2 else 2):
-        sl_in, sl_cmp = [], []
-        for d in range(nd):
-            hi = (corner >> d) & 1
-            if hi:
-                sl_in.append(slice(dims[d] - K, dims[d]))
-            else:
-                sl_in.append(slice(0, K))
-        sub = np.ascontiguousarray(a[tuple(sl_in)])
-        if min(sub.shape) < K:
-            sub = a
-        ref = oracle.run(kind, sub, T, hhc.FUSED)
-        for d in range(nd):
-            hi = (corner >> d) & 1
-            sl_cmp.append(slice(K - 4, K) if hi else slice(0, 4))
-        g = got[tuple(sl_in)][tuple(sl_cmp)]
-        r = ref[tuple(sl_cmp)]
-        assert_bits(np.ascontiguousarray(g), np.ascontiguousarray(r), f"{cfg} corner {corner}")
-    # global invariant: values stay in [min, max] of the input (positive weights / gradient)
-    assert got.min() >= a.min() - 1e-6 and got.max() <= a.max() + 1e-6
-
-
-@pytest.mark.parametrize("cfg,kind,dims,T", FULL[1:])
-def test_full_size_closed_forms(cfg, kind, dims, T):
-    """Whole-grid checks at full size: affine fields are exact fixed points
-    (dyadic kinds and Gradient), and a sine mode decays by lambda^T."""
-    tile = bench_tile(cfg)
-    nd = len(dims)
-    aff = np.ones(dims, np.float32)
-    for d, c in zip(range(nd), (1.0, 2.0, 3.0)):
-        aff += (c * np.arange(dims[d], dtype=np.float32)).reshape([-1 if e == d else 1 for e in range(nd)])
-    got = gpu_run(kind, aff, T, tile, hhc.FUSED)
-    assert np.array_equal(got, aff), cfg
-    if kind == hhc.GRADIENT2D:
-        return
-    offs, w = oracle.stencil_info(kind)
-    p = (3, 5, 2)[:nd]
-    th = np.array([math.pi * p[d] / (dims[d] - 1) for d in range(nd)])
-    lam = sum(float(wj) * np.prod(np.cos(th * o[:nd])) for o, wj in zip(offs, w))
-    sines = []
-    for d in range(nd):
-        sv = np.sin(th[d] * np.arange(dims[d]))
-        sv[0] = sv[-1] = 0.0
-        sines.append(sv)
-    rest = sines[1][:, None] * sines[2][None, :] if nd == 3 else sines[1]
-    u32 = (sines[0].reshape([-1] + [1] * (nd - 1)) * rest[None]).astype(np.float32)
-    got = gpu_run(kind, u32, T, tile, hhc.FUSED)
-    del u32
-    tol = (4 * T * len(w) + 2) * 2.0 ** -24
-    for x0 in range(0, dims[0], 64):                  # slab-wise, bounded host memory
-        ex = (lam ** T) * sines[0][x0:x0 + 64].reshape([-1] + [1] * (nd - 1)) * rest[None]
-        assert np.max(np.abs(got[x0:x0 + 64].astype(np.float64) - ex)) <= tol, (cfg, lam, x0)
 
 
 @pytest.mark.parametrize("kind,dims,T,tT,nslab", [

@@ -105,24 +105,94 @@ def test_special_case_wide_vector_units():
         assert math.isclose(mo.c_eq15(tS1, tT, tS2, hw), tT * (hw.C_iter + hw.tau_sync), rel_tol=1e-12)
 
 
-def test_k_branches():
-    """Eq. 16: k = 1 gives (m'+c)*N2, k > 1 gives m' + k*max(m',c)*N2."""
-    hw = mo.gtx980(2)
-    S, T = (4096, 4096), 1024
-    # a tile with Mtile just under 48 KB -> k = 2; shrink MSM to force k = 1
-    tile = (8, 8, 256, 0)
-    t2 = mo.talg(2, S, T, tile, hw)
-    hw1 = mo.gtx980(2)
-    hw1.MSM = 48 * 1024
-    t1 = mo.talg(2, S, T, tile, hw1)
-    Nw, w = mo.Nw_eq3(T, 8), mo.w_eq5(4096, 8, 8)
-    mi = 256 * (8 + 16)
-    mp = 2 * mi * hw.L + 2 * hw.tau_sync
-    c = mo.c_eq15(8, 8, 256, hw)
-    N2 = math.ceil((4096 + 8) / 256)
-    assert math.isclose(t1, Nw * hw.T_sync + Nw * (mp + c) * N2 * math.ceil(w / 16), rel_tol=1e-12)
-    assert math.isclose(t2, Nw * hw.T_sync + Nw * (mp + 2 * max(mp, c) * N2) * math.ceil(math.ceil(w / 2) / 16),
-                        rel_tol=1e-12)
+def test_k_equals_1_hand_example():
+    """Eq. 16's k = 1 branch (Tprism = (m' + c) * N2), worked by hand on a
+    B200-sized shared memory (MSM = 228 KB, Mblock = 227 KB) with round
+    constants L = 1e-12 s/word, tau_sync = 1e-9 s, T_sync = 2e-6 s,
+    Citer = 1e-8 s; Heat-2D, S1 = S2 = 8192, T = 1024, tile (16, 20, 512):
+      Nw = 2*64 + 1 = 129                (Eq. 3, T mod tT = 0 -> eps = 1)
+      w = ceil(8192 / 56) = 147          (Eq. 5)
+      Mtile = 2*37*529 = 39146 words = 156584 B  (Eq. 19)
+      k = min(floor(233472 / 156584), 32) = 1    (Eq. 11)
+      mi = mo = 512*(20+32) = 26624      (Eq. 13)
+      m' = 53248e-12 + 2e-9 = 5.5248e-8 s        (Eq. 14)
+      c = 2e-8 * sum_{x=20,22..34} ceil(512x/128) + 16e-9
+        = 2e-8 * 4*216 + 1.6e-8 = 1.7296e-5 s   (Eq. 15)
+      N2 = ceil(8208/512) = 17
+      Tprism = (m' + c) * N2 = 1.7351248e-5 * 17 = 2.94971216e-4 s  (Eq. 16, k = 1)
+      rounds = ceil(ceil(147/1)/148) = 1
+      Talg = 129*2e-6 + 129*2.94971216e-4*1 = 0.038309286864 s  (Eq. 17)"""
+    hw = mo.HW(nSM=148, nV=128, MTBSM=32, RSM=65536, MSM=228 * 1024, Mblock=227 * 1024, L=1e-12,
+               tau_sync=1e-9, T_sync=2e-6, C_iter=1e-8)
+    assert mo.Nw_eq3(1024, 16) == 129
+    assert mo.w_eq5(8192, 20, 16) == 147
+    assert math.isclose(mo.c_eq15(20, 16, 512, hw), 1.7296e-5, rel_tol=1e-12)
+    t = mo.talg(2, (8192, 8192), 1024, (16, 20, 512, 0), hw)
+    assert math.isclose(t, 0.038309286864, rel_tol=1e-11), t
+    # one more MTBSM-limited block per SM would be k = 2: the k > 1 branch differs
+    hw.MSM = 2 * 156584
+    assert not math.isclose(mo.talg(2, (8192, 8192), 1024, (16, 20, 512, 0), hw), 0.038309286864, rel_tol=1e-6)
+
+
+def test_hand_worked_heat3d_gtx980_paper():
+    """The PAPER-literal 3D model (Eqs. 20-30) worked by
+    hand on the GTX 980 constants (Tables 2-4: nSM = 16, nV = 128, MTBSM = 32,
+    MSM = 96 KB, Mblock = 48 KB, L = 7.36e-3 s/GB -> 2.944e-11 s/word,
+    tau_sync = 7.96e-10 s, T_sync = 9.24e-7 s, Citer(Heat3D) = 1.55e-7 s) for
+    Heat-3D, S1 = S2 = S3 = 384 (a size of P:L1179-1195), T = 128, tile
+    (tT, tS1, tS2, tS3) = (4, 4, 4, 32):
+      Nw = 2*32 + 1 = 65                  (Eq. 20 with Eq. 3's eps, T mod tT = 0)
+      w = ceil(384 / 12) = 32             (Eq. 22, pitch 2tS1 + tT, reading M2)
+      mi = mo = 4*32*(4+8) = 1536 words   (Eq. 24)
+      m' = 3072*2.944e-11 + 2*7.96e-10 = 9.203168e-8 s            (Eq. 25)
+      wtile = 4 + 4 - 2 = 6;  x = 4, 6:  ceil(4*128/128) + ceil(6*128/128) = 10
+      c = 2*1.55e-7*10 + 4*7.96e-10 = 3.103184e-6 s               (Eq. 27)
+      Mtile = 2*9*9*37 = 5994 words = 23976 B <= 48 KB            (reading M3)
+      k = min(floor(98304/23976), 32) = 4                          (Eq. 11)
+      Nsslabs = ceil((388/4)*(388/32)) = ceil(97*12.125) = 1177   (Eq. 23 as printed)
+      zeta = max(m', c) = c
+      Tslab = m' + k*zeta*Nsslabs = 9.203168e-8 + 4*3.103184e-6*1177
+            = 0.01460988230368 s                                   (Eq. 29)
+      rounds = ceil(ceil(32/4)/16) = 1
+      Talg = 65*9.24e-7 + 65*0.01460988230368*1 = 0.9497024097392 s  (Eq. 30)"""
+    hw = mo.gtx980(4)
+    assert mo.Nw_eq3(128, 4) == 65
+    assert mo.w_eq5(384, 4, 4) == 32
+    assert math.isclose(mo.c_eq15(4, 4, 4 * 32, hw), 3.103184e-6, rel_tol=1e-12)
+    t = mo.talg(3, (384, 384, 384), 128, (4, 4, 4, 32), hw)
+    assert math.isclose(t, 0.9497024097392, rel_tol=1e-11), t
+
+
+def test_multi_gpu_model_hand_example():
+    """Reading M7 (not in the paper) worked by hand with a stub single-GPU time:
+    PAPER geometry on the k = 1 hardware above is replaced by the closed form
+    of a constant per-row cost, so only M7's own arithmetic is checked.
+    G = 4, S1 = 1000 -> own = 250, e = 2, g = tT = 8, T = 20 -> tiles 8, 8, 4;
+    inner S2 = 100 -> T_exch = 8*100*4 B / 1e9 B/s + 1e-6 = 4.2e-6 s."""
+    calls = []
+
+    def fake(nd, S, T, tile, hw):
+        calls.append((S[0], T))
+        return 1e-6 * S[0] * T                       # 1 us per row-step
+
+    orig = mo.talg_single
+    mo.talg_single = fake
+    try:
+        hw = mo.gtx980(2)
+        hw.n_gpus, hw.link_Bps, hw.link_lat = 4, 1e9, 1e-6
+        # plain: (266*8 + 266*8 + 266*4) us + 3 * 4.2 us
+        t = mo.talg(2, (1000, 100), 20, (8, 8, 64, 0), hw)
+        assert math.isclose(t, 1e-6 * 266 * 20 + 3 * 4.2e-6, rel_tol=1e-12), t
+        # overlap: interior 250 rows, 2 edge sub-slabs of 24 rows, exchange hidden (250*Tt us >> 4.2 us)
+        hw.dist_overlap = 1
+        t = mo.talg(2, (1000, 100), 20, (8, 8, 64, 0), hw)
+        assert math.isclose(t, 1e-6 * (250 + 2 * 24) * 20, rel_tol=1e-12), t
+        # G = 2: one neighbour
+        hw.n_gpus, hw.dist_overlap = 2, 0
+        t = mo.talg(2, (1000, 100), 20, (8, 8, 64, 0), hw)
+        assert math.isclose(t, 1e-6 * 508 * 20 + 3 * 4.2e-6, rel_tol=1e-12), t
+    finally:
+        mo.talg_single = orig
 
 
 def test_infeasible_and_invalid_tiles():
