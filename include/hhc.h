@@ -16,9 +16,9 @@
  *   model_select_tile  -- Eq. 31 solved by exhaustive enumeration, plus the
  *                         "within 10% of Talg_min" candidates.
  *   stencil_run_planes -- one time tile of the slab-decomposed multi-GPU run
- *                         (BASELINE.json north_star; not in the paper): the
- *                         ghost exchange is torch.distributed P2P over NCCL in
- *                         the Python binding, see DESIGN.md §Multi-GPU.
+ *   stencil_run_dist   -- the multi-GPU slab path with its NCCL ghost exchange
+ *                         (BASELINE.json north_star; not in the paper), see
+ *                         DESIGN.md §8.
  *
  * Conventions (all functions):
  *   - Sizes are int64.  Arrays are fp32, contiguous, row-major, S1 OUTERMOST,
@@ -56,7 +56,7 @@ typedef enum {
     STENCIL_ETILE = -2,    /* tile violates Eq. 31's integrality or the smem limit   */
     STENCIL_ENOMEM = -3,   /* device or host allocation failed                        */
     STENCIL_ECUDA = -4,    /* a CUDA runtime error (sticky until stencil_destroy)     */
-    STENCIL_ENCCL = -5,    /* reserved: NCCL error (multi-GPU exchange is in Python)  */
+    STENCIL_ENCCL = -5,    /* NCCL missing or an NCCL call failed (multi-GPU path)    */
     STENCIL_ENODEV = -6    /* no usable sm_100 device                                 */
 } stencil_status;
 
@@ -181,6 +181,56 @@ int stencil_microbench(int which, stencil_kind kind, int ndims, const int64_t* d
  * dims[0] (ghost-extended slabs).  Stream-ordered like stencil_run. */
 int stencil_run_planes(stencil_t h, int64_t rows, float* plane0, float* plane1, int64_t T,
                        stencil_tile tile, int threads, void* cuda_stream);
+
+/* ---- Multi-GPU slab path (BASELINE.json north_star -- the
+ * paper is single-GPU, so no PAPER.md passage defines it; its time model is
+ * DESIGN.md reading M7).  One process per GPU.  The interior S1 rows are cut
+ * into `world` slabs of own = ceil((S1-2)/world) rows; every time tile of tT
+ * steps each rank exchanges g = tT ghost rows with rank -/+ 1 by ncclSend /
+ * ncclRecv inside ncclGroupStart/End (point to point, no collective), then runs
+ * the HHC rows (stencil_run_planes) on its ghost-extended slab.  NCCL is
+ * dlopen'ed (libnccl.so.2, the copy already loaded by the process if any). */
+
+/* ncclGetUniqueId into id[128] (rank 0 calls it; the caller broadcasts it, e.g.
+ * with torch.distributed).  STENCIL_ENCCL if NCCL cannot be loaded. */
+int stencil_dist_get_unique_id(unsigned char id[128]);
+
+/* ncclCommInitRank on `device` (made current).  *comm receives an opaque
+ * communicator owned by the library (free with stencil_dist_destroy); it also
+ * owns the ghost-extended planes, the edge buffers and a second stream.
+ * world = 1 needs no id and no NCCL. */
+int stencil_dist_init(const unsigned char id[128], int rank, int world, int device, void** comm);
+
+/* 0 (default): exchange, then the whole ghost-extended slab per tile (2g
+ * redundant rows); 1: edge sub-slabs (3g rows per side) first on the second
+ * stream, their owned rows sent at once, the ghost-free interior overlapped
+ * with the exchange (6g redundant rows; used only if every slab holds >= 2g rows). */
+int stencil_dist_set_overlap(void* comm, int overlap);
+
+/* Synchronises the device, frees the communicator and its buffers.  NULL ok. */
+void stencil_dist_destroy(void* comm);
+
+/* Host-only slab geometry (no device needed): part[0..5] = owned rows [r0, r1),
+ * ghost-extended rows [e0, e1), rows the caller's slab holds [held_lo, held_hi)
+ * (owned + the physical ring row on rank 0 / world-1), global row indices.
+ * STENCIL_ETILE if a slab is thinner than g (world > 1). */
+int stencil_dist_partition(int64_t S1, int rank, int world, int64_t g, int64_t part[6]);
+
+/* A_T on this rank's slab.  h was created with the GLOBAL dims.  d_in_slab and
+ * d_out_slab (device, caller-owned, no overlap) hold rows [held_lo, held_hi) of
+ * the global array (stencil_dist_partition with g = tile.t).  Every rank calls
+ * it with the same T, tile and threads.  Stream-ordered on cuda_stream (the
+ * NCCL operations too); returns before completion.  stencil_last_launches(h)
+ * then counts this rank's kernel launches. */
+int stencil_run_dist(stencil_t h, void* comm, const float* d_in_slab, float* d_out_slab, int64_t T,
+                     stencil_tile tile, int threads, void* cuda_stream);
+
+/* The same per-rank phases for `world` virtual ranks of ONE device in lock
+ * step, the ghost exchange done by device copies from the neighbour's buffers:
+ * full-grid d_in/d_out (every rank's held rows are written).  Synchronises.
+ * The single-GPU test of the slab path. */
+int stencil_run_dist_local(stencil_t h, int world, const float* d_in, float* d_out, int64_t T,
+                           stencil_tile tile, int threads, int overlap, void* cuda_stream);
 
 /* Measurement helper (bench.py roofline): run like stencil_run but without the
  * CUDA graph, with a CUDA event pair around every hexagon-row launch on

@@ -125,6 +125,15 @@ def load(build_if_missing: bool = False):
     lib.model_select_wavefront_tile.argtypes = [ctypes.c_int, ctypes.c_int, i64p, ctypes.c_int64,
                                                 P(model_hw_params), ctypes.c_double, P(stencil_tile),
                                                 P(stencil_tile), ctypes.c_int, P(ctypes.c_int)]
+    lib.stencil_dist_get_unique_id.argtypes = [ctypes.c_char_p]
+    lib.stencil_dist_init.argtypes = [ctypes.c_char_p, ctypes.c_int, ctypes.c_int, ctypes.c_int, P(vp)]
+    lib.stencil_dist_set_overlap.argtypes = [vp, ctypes.c_int]
+    lib.stencil_dist_destroy.argtypes = [vp]
+    lib.stencil_dist_destroy.restype = None
+    lib.stencil_dist_partition.argtypes = [ctypes.c_int64, ctypes.c_int, ctypes.c_int, ctypes.c_int64, i64p]
+    lib.stencil_run_dist.argtypes = [vp, vp, vp, vp, ctypes.c_int64, stencil_tile, ctypes.c_int, vp]
+    lib.stencil_run_dist_local.argtypes = [vp, ctypes.c_int, vp, vp, ctypes.c_int64, stencil_tile, ctypes.c_int,
+                                           ctypes.c_int, vp]
     _lib = lib
     return lib
 
@@ -300,6 +309,46 @@ def stencil_tile_occupancy(kind: int, tile, threads: int = 0, mode: int = FUSED)
     return k.value
 
 
+def stencil_dist_get_unique_id() -> bytes:
+    buf = ctypes.create_string_buffer(128)
+    _check(load().stencil_dist_get_unique_id(buf), "stencil_dist_get_unique_id")
+    return buf.raw
+
+
+def stencil_dist_init(uid, rank: int, world: int, device: int):
+    """NCCL communicator of this rank (opaque); uid = rank 0's stencil_dist_get_unique_id()."""
+    comm = ctypes.c_void_p()
+    _check(load().stencil_dist_init(uid if uid else None, int(rank), int(world), int(device), ctypes.byref(comm)),
+           "stencil_dist_init")
+    return comm
+
+
+def stencil_dist_set_overlap(comm, overlap: int):
+    _check(load().stencil_dist_set_overlap(comm, int(overlap)), "stencil_dist_set_overlap")
+
+
+def stencil_dist_destroy(comm):
+    load().stencil_dist_destroy(comm)
+
+
+def stencil_dist_partition(S1: int, rank: int, world: int, g: int):
+    """(r0, r1, e0, e1, held_lo, held_hi) of one rank's slab (host only)."""
+    out = (ctypes.c_int64 * 6)()
+    _check(load().stencil_dist_partition(int(S1), int(rank), int(world), int(g), out), "stencil_dist_partition")
+    return tuple(out)
+
+
+def stencil_run_dist(h, comm, d_in_slab, d_out_slab, T: int, tile, threads: int = 0, stream=None):
+    _check(load().stencil_run_dist(h.handle, comm, _ptr(d_in_slab), _ptr(d_out_slab), int(T), make_tile(tile),
+                                   int(threads), _stream(stream)), "stencil_run_dist")
+
+
+def stencil_run_dist_local(h, world: int, d_in, d_out, T: int, tile, threads: int = 0, overlap: int = 0,
+                           stream=None):
+    _check(load().stencil_run_dist_local(h.handle, int(world), _ptr(d_in), _ptr(d_out), int(T), make_tile(tile),
+                                         int(threads), int(overlap), _stream(stream)), "stencil_run_dist_local")
+
+
 def stencil_plan_info(dims, T: int, tile):
     d, nd = _dims(dims)
     out = [ctypes.c_int64() for _ in range(4)]
@@ -326,4 +375,6 @@ EXPORTED_SYMBOLS = ["stencil_create", "stencil_destroy", "stencil_run", "stencil
                     "stencil_run_planes", "model_predict", "model_select_tile", "stencil_tile_resources", "stencil_tile_occupancy",
                     "stencil_plan_info", "stencil_microbench", "stencil_strerror", "stencil_last_launches",
                     "stencil_profile", "stencil_run_wavefront", "stencil_wavefront_info",
-                    "model_predict_wavefront", "model_select_wavefront_tile"]
+                    "model_predict_wavefront", "model_select_wavefront_tile", "stencil_dist_get_unique_id",
+                    "stencil_dist_init", "stencil_dist_set_overlap", "stencil_dist_destroy", "stencil_dist_partition",
+                    "stencil_run_dist", "stencil_run_dist_local"]

@@ -11,7 +11,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libhhc.so")
 BUILD = os.path.join(HERE, "build")
-SOURCES = ["hhc_kernels.cu", "wave_kernels.cu", "hhc_api.cu", "microbench.cu", "model.cpp"]
+SOURCES = ["hhc_kernels.cu", "wave_kernels.cu", "hhc_api.cu", "hhc_dist.cu", "microbench.cu", "model.cpp"]
 HEADERS = ["hhc_internal.h", "hhc_device.cuh", os.path.join("..", "..", "include", "hhc.h")]
 
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")

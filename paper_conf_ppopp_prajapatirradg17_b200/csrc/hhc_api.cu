@@ -95,6 +95,7 @@ struct stencil_s {
     int compute_only = 0;
     int occ = 1;
     int envJ = 0;               // HHC_J read once at create (experiments; 0 = library rule)
+    int maxJ = 0;               // > 0: cap on the 3D blocks per slab (1 = never wait on flags)
 
     int64_t nelem() const { return dims[0] * dims[1] * dims[2]; }
 };
@@ -319,6 +320,7 @@ static int choose_J(stencil_t h, const RowPlan& r) {
     const int cap = std::max(1, h->nsm * std::max(h->occ, 1) / std::max(r.w, 1));
     int J = std::max(1, std::min(r.n2, cap));
     if (h->envJ > 0) J = std::max(1, std::min({h->envJ, r.n2, cap}));
+    if (h->maxJ > 0) J = std::min(J, h->maxJ);
     return J;
 }
 
@@ -684,4 +686,30 @@ extern "C" int stencil_microbench(int which, stencil_kind kind, int ndims, const
 
 namespace hhc {
 void set_compute_only(stencil_t h, int on) { if (h) h->compute_only = on; }
+
+void set_last_launches(stencil_t h, int64_t n) { if (h) h->last_launches = n; }
+
+void handle_info(stencil_t h, int* kind, int* ndims, int64_t* dims, int* device) {
+    *kind = h->kind;
+    *ndims = h->ndims;
+    for (int d = 0; d < 3; ++d) dims[d] = h->dims[d];
+    *device = h->device;
+}
+
+// A handle with h's stencil (kind, weights, c, mode) on other extents; maxJ > 0
+// caps its 3D blocks per slab (the multi-GPU edge runs use 1: they never spin on
+// progress flags, so they can share the GPU with a J-pipelined interior run).
+int handle_clone(stencil_t h, const int64_t* dims, int maxJ, stencil_t* out) {
+    float co[kMaxPts + 1];
+    int n = 0;
+    if (h->kind == STENCIL_GRADIENT2D) {
+        co[n++] = h->kappa;
+    } else {
+        for (int j = 0; j < h->npts; ++j) co[n++] = h->w[j];
+        co[n++] = h->c;
+    }
+    const int rc = stencil_create((stencil_kind)h->kind, h->ndims, dims, co, n, h->mode, out);
+    if (rc == STENCIL_OK) (*out)->maxJ = maxJ;
+    return rc;
+}
 }

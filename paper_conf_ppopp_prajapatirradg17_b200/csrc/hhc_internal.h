@@ -61,6 +61,9 @@ void launch_copy_ring(const float* in, float* out, int64_t S1, int64_t S2, int64
 void launch_copy_full(const float* in, float* out, int64_t n, void* stream);
 
 void set_compute_only(stencil_t h, int on);
+void set_last_launches(stencil_t h, int64_t n);
+void handle_info(stencil_t h, int* kind, int* ndims, int64_t* dims, int* device);
+int handle_clone(stencil_t h, const int64_t* dims, int maxJ, stencil_t* out);
 
 // ---- wavefront-parallel Jacobi-1D (reading W1)
 // Parallelogram tiles in skewed coordinates x' = x + t: tile (i, j) computes the

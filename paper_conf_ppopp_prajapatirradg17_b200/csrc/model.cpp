@@ -102,13 +102,14 @@ int default_threads(int nd, const stencil_tile& t) {
 
 // Eq. 11's k under the CUDA occupancy rules (reading M4): shared memory per block
 // plus the 1 KB the driver reserves per block, registers allocated per warp in
-// units of 256, at most MTBSM blocks and max_threads_sm threads per SM.
+// units of 256 from one of the 4 sub-partition register files (RSM/4 each), at
+// most MTBSM blocks and max_threads_sm threads per SM.
 int64_t k_exact(int64_t Mtile, int64_t threads, const model_hw_params& hw) {
     const int64_t maxthr = hw.max_threads_sm > 0 ? hw.max_threads_sm : 2048;
     int64_t k = std::min<int64_t>({hw.m_sm_bytes / (Mtile + 1024), (int64_t)hw.mtb_sm, maxthr / threads});
     if (hw.regs_per_thread > 0) {
         const int64_t per_warp = cdiv(32 * (int64_t)hw.regs_per_thread, 256) * 256;
-        k = std::min<int64_t>(k, (hw.r_sm / per_warp) / cdiv(threads, 32));
+        k = std::min<int64_t>(k, 4 * ((hw.r_sm / 4) / per_warp) / cdiv(threads, 32));
     }
     return k;
 }

@@ -36,14 +36,34 @@ KINDS = [hhc.JACOBI2D_5PT, hhc.HEAT2D_9PT, hhc.LAPLACIAN2D_5PT, hhc.GRADIENT2D, 
          hhc.LAPLACIAN3D_27PT, hhc.JACOBI1D_3PT]
 
 
+def kernel_regs(kind: int, tile=None, threads: int = 0) -> int:
+    """Registers per thread of the kernel the library launches (Eq. 11's Rtile,
+    reading M4) from cudaFuncGetAttributes; `tile` None = the generic-width
+    instantiation (2D tS2 = 64).  0 without a device."""
+    nd = hhc.KIND_NDIMS[kind]
+    if tile is None:
+        tile = {1: (8, 64, 0, 0), 2: (8, 4, 64, 0), 3: (4, 2, 2, 32)}[nd]
+    try:
+        return hhc.stencil_tile_resources(nd, tile, threads, kind=kind)[2]
+    except hhc.StencilError:
+        return 0
+
+
 def b200_hw(cal: dict | None, kind: int, geometry: int, threads: int = 0,
-            leff: bool = False) -> "hhc.model_hw_params":
-    """Table 2 analogue for B200 plus calibrated Table 3/4 constants."""
+            leff: bool = False, tile=None) -> "hhc.model_hw_params":
+    """Table 2 analogue for B200 plus calibrated Table 3/4 constants; the
+    register count of the kernel (for `tile`, else the generic instantiation)
+    bounds k in EXACT (Eq. 11, reading M4): live from the device, else the
+    calibration file's record."""
     import torch
     props = torch.cuda.get_device_properties(0) if torch.cuda.is_available() else None
     n_sm = props.multi_processor_count if props else 148
     hw = hhc.make_hw(n_sm=n_sm, n_v=128, mtb_sm=32, r_sm=65536, m_sm_bytes=228 * 1024,
                      m_block_bytes=227 * 1024, geometry=geometry, threads=threads, max_threads_sm=2048)
+    regs = kernel_regs(kind, tile, threads) if props else 0
+    if not regs and cal:
+        regs = int((cal.get("regs_per_thread") or {}).get(str(kind), 0))
+    hw.regs_per_thread = regs
     if cal:
         hw.L_s_per_word = cal["L_s_per_word"]
         hw.tau_sync_s = cal["tau_sync_s"]
@@ -142,6 +162,7 @@ def calibrate(args):
         out["L_s_per_GB"] = out["L_s_per_word"] / 4e-9
         out["tau_sync_s"] = hhc.stencil_microbench(1, threads=256)
         out["T_sync_s"] = hhc.stencil_microbench(2)
+        out["regs_per_thread"] = {str(k): kernel_regs(k) for k in KINDS}
     rnd = random.Random(2017)
     citer, samples, fits, insts, raw, full, full_all = {}, {}, {}, [], {}, [], {}
     for kind in kinds:
@@ -298,10 +319,11 @@ def sweep(args):
             continue
         p = {"tile": list(tile), "threads": threads, "texec": te}
         for geom, name in ((hhc.PAPER, "talg_paper"), (hhc.EXACT, "talg_exact")):
-            p[name] = hhc.model_predict(kind, dims, T, tile, b200_hw(cal, kind, geom, threads))
+            p[name] = hhc.model_predict(kind, dims, T, tile, b200_hw(cal, kind, geom, threads, tile=tile))
         if (cal.get("exact_leff") or {}).get(str(kind)):
             p["talg_exact_leff"] = hhc.model_predict(kind, dims, T, tile,
-                                                     b200_hw(cal, kind, hhc.EXACT, threads, leff=True))
+                                                     b200_hw(cal, kind, hhc.EXACT, threads, leff=True,
+                                                             tile=tile))
         pts.append(p)
         print(json.dumps(p), flush=True)
     best = min(pts, key=lambda p: p["texec"])
@@ -324,7 +346,7 @@ def sweep(args):
                                      "n_within_10pct": len(cands)}
         except hhc.StencilError as e:
             res[f"argmin_{name}"] = {"error": str(e)}
-    out = args.out or os.path.join(ROOT, "profiles", f"sweep_{args.config}_r01.json")
+    out = args.out or os.path.join(ROOT, "profiles", f"sweep_{args.config}_r02.json")
     with open(out, "w") as f:
         json.dump(res, f, indent=1)
     print(json.dumps({k: v for k, v in res.items() if k != "points"}))
@@ -358,7 +380,7 @@ def select(args):
     win = min(meas, key=lambda m: m["texec"])
     res = {"config": args.config, "argmin": list(best), "argmin_threads": thr, "n_candidates": len(cands),
            "enumeration_seconds": t_sel, "measured": meas, "best_within": win}
-    out = args.out or os.path.join(ROOT, "profiles", f"select_{args.config}_r01.json")
+    out = args.out or os.path.join(ROOT, "profiles", f"select_{args.config}_r02.json")
     with open(out, "w") as f:
         json.dump(res, f, indent=1)
     print(json.dumps({k: v for k, v in res.items() if k != "measured"}))

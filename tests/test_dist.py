@@ -12,7 +12,7 @@ import torch.distributed as dist
 import torch.multiprocessing as mp
 
 import oracle
-from paper_conf_ppopp_prajapatirradg17_b200 import dist as hdist
+import slab_reference as hdist
 from synth import field
 
 
@@ -102,3 +102,20 @@ def test_partition_rules():
     assert s7.r1 == 8193 and s7.e1 == 8194 and s7.held[1] == 8194
     with pytest.raises(ValueError):
         hdist.partition(40, 8, 0, 16)            # slabs thinner than the ghost depth
+
+
+def test_product_partition_matches_reference():
+    """The library's slab geometry (stencil_dist_partition, used by
+    stencil_run_dist) equals the algorithm reference tested above."""
+    import paper_conf_ppopp_prajapatirradg17_b200 as hhc
+    for S1 in (20, 41, 70, 1000, 8194, 16386):
+        for world in (1, 2, 3, 4, 7, 8):
+            for g in (2, 4, 8, 16, 32):
+                for rank in range(world):
+                    try:
+                        s = hdist.partition(S1, world, rank, g)
+                    except ValueError:
+                        with pytest.raises(hhc.StencilError):
+                            hhc.stencil_dist_partition(S1, rank, world, g)
+                        continue
+                    assert hhc.stencil_dist_partition(S1, rank, world, g) == (s.r0, s.r1, s.e0, s.e1) + s.held

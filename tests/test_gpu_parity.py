@@ -139,49 +139,47 @@ def test_parity_mid_size(kind, dims, T, tile):
     assert max_rel(gpu_run(kind, a, T, tile, hhc.FUSED), plain) <= 1e-5
 
 
-@pytest.mark.parametrize("kind,dims,T,tT,nslab", [
-    (hhc.HEAT2D_9PT, (131, 150), 37, 8, 3),
-    (hhc.GRADIENT2D, (90, 77), 21, 4, 2),
-    (hhc.HEAT3D_7PT, (40, 30, 70), 11, 4, 2),
-    (hhc.LAPLACIAN3D_27PT, (45, 22, 40), 9, 2, 3),
+@pytest.mark.parametrize("kind,dims,T,tT,world,overlap", [
+    (hhc.HEAT2D_9PT, (131, 150), 37, 8, 3, 0),
+    (hhc.HEAT2D_9PT, (2 * 160 + 2, 300), 37, 8, 2, 1),
+    (hhc.GRADIENT2D, (90, 77), 21, 4, 2, 0),
+    (hhc.GRADIENT2D, (3 * 60 + 2, 130), 21, 4, 3, 1),
+    (hhc.JACOBI2D_5PT, (4 * 40 + 2, 70), 19, 6, 4, 1),
+    (hhc.HEAT3D_7PT, (40, 30, 70), 11, 4, 2, 0),
+    (hhc.HEAT3D_7PT, (2 * 40 + 2, 30, 70), 13, 4, 2, 1),
+    (hhc.LAPLACIAN3D_27PT, (45, 22, 40), 9, 2, 3, 0),
+    (hhc.LAPLACIAN3D_27PT, (3 * 20 + 2, 22, 40), 9, 2, 3, 1),
 ])
-def test_virtual_slabs_run_planes(kind, dims, T, tT, nslab):
-    """The multi-GPU time-tile loop (dist.partition + stencil_run_planes) with
-    `nslab` virtual ranks on one GPU; ghosts are exchanged by device copies in
-    the same pattern as dist.exchange.  Owned rows must equal the oracle."""
-    from paper_conf_ppopp_prajapatirradg17_b200 import dist as hdist
-    a = field(99, dims)
+def test_dist_local_virtual_ranks(kind, dims, T, tT, world, overlap):
+    """The library's multi-GPU slab path (hhc_dist.cu: partition, ghost-extended
+    planes, per-tile exchange, plain or overlapped edge/interior phases) with
+    `world` virtual ranks of this GPU (stencil_run_dist_local; device copies in
+    place of ncclSend/ncclRecv).  Every held row must equal the oracle."""
+    a = field(99 + overlap, dims)
     tile = (tT, 3, 32) if len(dims) == 2 else (tT, 2, 3, 32)
-    slabs = [hdist.partition(dims[0], nslab, r, tT) for r in range(nslab)]
-    hs = [hhc.stencil_create(kind, (s.rows,) + dims[1:]) for s in slabs]
-    p0 = [torch.from_numpy(np.ascontiguousarray(a[s.e0:s.e1])).to(DEV) for s in slabs]
-    p1 = [torch.empty_like(x) for x in p0]
-    cur = list(p0)
-    done = 0
-    while done < T:
-        Tt = min(tT, T - done)
-        for r, s in enumerate(slabs):            # ghost exchange (the dist.exchange pattern)
-            lo, hi = s.r0 - s.e0, s.r1 - s.e0
-            if r > 0:
-                sp = slabs[r - 1]
-                cur[r][lo - tT:lo] = cur[r - 1][sp.r1 - sp.e0 - tT:sp.r1 - sp.e0]
-            if r < nslab - 1:
-                sn = slabs[r + 1]
-                cur[r][hi:hi + tT] = cur[r + 1][sn.r0 - sn.e0:sn.r0 - sn.e0 + tT]
-        torch.cuda.synchronize()
-        for r in range(nslab):
-            other = p1[r] if cur[r] is p0[r] else p0[r]
-            hhc.stencil_run_planes(hs[r], slabs[r].rows, cur[r], other, Tt, tile)
-            cur[r] = cur[r] if Tt % 2 == 0 else other
-        torch.cuda.synchronize()
-        done += Tt
-    exp = oracle.run(kind, a, T, hhc.FUSED)
-    for r, s in enumerate(slabs):
-        lo, hi = s.held
-        got = cur[r][lo - s.e0:hi - s.e0].cpu().numpy()
-        assert_bits(np.ascontiguousarray(got), np.ascontiguousarray(exp[lo:hi]), f"slab {r}")
+    s = hhc.stencil_create(kind, dims)
+    d_in = torch.from_numpy(a).to(DEV)
+    d_out = torch.full_like(d_in, float("nan"))
+    hhc.stencil_run_dist_local(s, world, d_in, d_out, T, tile, 0, overlap)
+    assert hhc.stencil_last_launches(s) > 0
+    hhc.stencil_destroy(s)
+    assert_bits(d_out.cpu().numpy(), oracle.run(kind, a, T, hhc.FUSED), f"world {world} overlap {overlap}")
 
 
+def test_dist_world1_nccl_free():
+    """stencil_run_dist on a world-1 communicator (no NCCL needed): the slab is
+    the whole grid."""
+    dims, T, tile = (70, 90), 13, (4, 3, 32)
+    a = field(5, dims)
+    comm = hhc.stencil_dist_init(None, 0, 1, 0)
+    s = hhc.stencil_create(hhc.HEAT2D_9PT, dims)
+    d_in = torch.from_numpy(a).to(DEV)
+    d_out = torch.empty_like(d_in)
+    hhc.stencil_run_dist(s, comm, d_in, d_out, T, tile)
+    torch.cuda.synchronize()
+    hhc.stencil_destroy(s)
+    hhc.stencil_dist_destroy(comm)
+    assert_bits(d_out.cpu().numpy(), oracle.run(hhc.HEAT2D_9PT, a, T, hhc.FUSED), "world 1")
 
 
 PAIR_TILES = [((2, 1, 256), 0), ((4, 3, 256), 64), ((8, 5, 512), 0), ((16, 4, 256), 128), ((6, 2, 768), 192),
@@ -235,88 +233,6 @@ def test_parity_1d_large_and_coeffs():
                     oracle.run(hhc.JACOBI1D_3PT, a[:20001], 33, mode, coeffs=coeffs), "1D coeffs")
     plain = oracle.run(hhc.JACOBI1D_3PT, a, 100, hhc.PLAIN)
     assert max_rel(gpu_run(hhc.JACOBI1D_3PT, a, 100, (32, 2048), hhc.FUSED), plain) <= 1e-5
-
-
-# ---- the overlapped multi-GPU loop (dist.run_slabs_overlap) on ONE GPU: virtual ranks in threads, each
-# with its own streams and handles, a queue-backed stand-in for torch.distributed's P2P (device copies
-# ordered by CUDA events).  Exercises the stream/event logic of the GPU path, not NCCL itself.
-class _Work:
-    def __init__(self, q, buf):
-        self.q, self.buf = q, buf
-
-    def wait(self):
-        t, ev = self.q.get(timeout=120)
-        torch.cuda.current_stream().wait_event(ev)
-        self.buf.copy_(t)
-
-
-class _FakeDist:
-    isend, irecv = "isend", "irecv"
-
-    class P2POp:
-        def __init__(self, op, tensor, peer):
-            self.op, self.tensor, self.peer = op, tensor, peer
-
-    def __init__(self, rank, board):
-        self.rank, self.board = rank, board
-
-    def batch_isend_irecv(self, ops):
-        works = []
-        for o in ops:
-            if o.op == "isend":
-                t = o.tensor.clone()
-                ev = torch.cuda.Event()
-                ev.record()
-                self.board[(self.rank, o.peer)].put((t, ev))
-            else:
-                works.append(_Work(self.board[(o.peer, self.rank)], o.tensor))
-        return works
-
-
-@pytest.mark.parametrize("kind,dims,T,tT,world", [
-    (hhc.HEAT2D_9PT, (2 * 160 + 2, 300), 37, 8, 2),
-    (hhc.GRADIENT2D, (3 * 60 + 2, 130), 21, 4, 3),
-    (hhc.HEAT3D_7PT, (2 * 40 + 2, 30, 70), 13, 4, 2),
-])
-def test_overlapped_slabs_gpu_streams(kind, dims, T, tT, world):
-    import queue
-    import threading
-    from paper_conf_ppopp_prajapatirradg17_b200 import dist as hdist
-    a = field(98, dims)
-    tile = (tT, 3, 32) if len(dims) == 2 else (tT, 2, 3, 32)
-    board = {(i, j): queue.Queue() for i in range(world) for j in range(world)}
-    out, errs = {}, []
-
-    def rank_main(r):
-        try:
-            torch.cuda.set_device(0)
-            s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
-            with torch.cuda.stream(s1):
-                slab = hdist.partition(dims[0], world, r, tT)
-                ext = (slab.rows,) + dims[1:]
-                h, he = hhc.stencil_create(kind, ext), hhc.stencil_create(kind, ext)
-                p0 = torch.from_numpy(np.ascontiguousarray(a[slab.e0:slab.e1])).to(DEV)
-                p1 = torch.empty_like(p0)
-                res = hdist.run_slabs_overlap(slab, p0, p1, T, tT, hdist.gpu_stepper(h, tile, 0, s1),
-                                              hdist.gpu_stepper(he, tile, 0, s2), _FakeDist(r, board), (s1, s2))
-                lo, hi = slab.held
-                out[r] = (lo, hi, res[lo - slab.e0:hi - slab.e0].cpu().numpy())
-                torch.cuda.synchronize()
-                hhc.stencil_destroy(h)
-                hhc.stencil_destroy(he)
-        except Exception as e:          # surfaced below
-            errs.append(e)
-
-    ts = [threading.Thread(target=rank_main, args=(r,)) for r in range(world)]
-    for t in ts:
-        t.start()
-    for t in ts:
-        t.join(300)
-    assert not errs, errs
-    exp = oracle.run(kind, a, T, hhc.FUSED)
-    for r in range(world):
-        lo, hi, got = out[r]
-        assert_bits(np.ascontiguousarray(got), np.ascontiguousarray(exp[lo:hi]), f"rank {r}")
 
 
 # ---- wavefront-parallel Jacobi-1D (reading W1): K3, one block per
