@@ -13,7 +13,7 @@ cmd=$1; shift
 case "$cmd" in
 tests)
   timeout 300 python __graft_entry__.py smoke > "$OUT/smoke.log" 2>&1; echo "smoke=$? $(tail -1 $OUT/smoke.log)"
-  timeout ${TEST_TIMEOUT:-2400} python -m pytest tests -m gpu -q -x ${PYTEST_ARGS} > "$OUT/gpu_tests.log" 2>&1
+  timeout ${TEST_TIMEOUT:-2400} python -m pytest tests -m gpu -q -x ${PYTEST_K:+-k "$PYTEST_K"} > "$OUT/gpu_tests.log" 2>&1
   echo "tests=$?"; tail -3 "$OUT/gpu_tests.log";;
 bench)
   for c in "$@"; do
