@@ -191,7 +191,8 @@ extern "C" void stencil_destroy(stencil_t h) {
 }
 
 // ---- tile validation (§8(b) validation rules; Eq. 31 integrality)
-static int check_tile(int ndims, stencil_tile t, int threads, int smem_limit, int* G_out, int* thr_out) {
+static int check_tile(int ndims, stencil_tile t, int threads, int smem_limit, int* G_out, int* thr_out,
+                      int kind = 0) {
     if (t.t < 2 || (t.t & 1) || t.s1 < 1) return STENCIL_ETILE;
     if (ndims == 1) {
         if (t.t > 1024 || t.s1 > 65536) return STENCIL_ETILE;
@@ -209,12 +210,12 @@ static int check_tile(int ndims, stencil_tile t, int threads, int smem_limit, in
     }
     if (t.t > 1024 || t.s1 > 4096 || t.s2 > 8192 || (ndims == 3 && t.s3 > 4096)) return STENCIL_ETILE;
     const int base = column_threads(ndims, t.s2, t.s3);
-    if (base > max_block_threads(ndims)) return STENCIL_ETILE;
+    if (base > max_block_threads(ndims, kind)) return STENCIL_ETILE;
     int G;
     if (threads == 0) {
         G = base <= 256 ? std::max(1, std::min(4, 256 / base)) : 1;
     } else {
-        if (threads < 0 || threads > max_block_threads(ndims) || threads % base) return STENCIL_EINVAL;
+        if (threads < 0 || threads > max_block_threads(ndims, kind) || threads % base) return STENCIL_EINVAL;
         G = threads / base;
     }
     const int64_t sm = smem_bytes(ndims, t.t, t.s1, t.s2, t.s3);
@@ -229,7 +230,7 @@ extern "C" int stencil_tile_resources(stencil_kind kind, int ndims, stencil_tile
     if (ndims < 1 || ndims > 3) return STENCIL_EINVAL;
     if (kind != 0 && kind_ndims_host(kind) != ndims) return STENCIL_EINVAL;
     int G, thr;
-    const int rc = check_tile(ndims, tile, threads, 227 * 1024, &G, &thr);
+    const int rc = check_tile(ndims, tile, threads, 227 * 1024, &G, &thr, kind);
     if (rc) return rc;
     if (smem) *smem = smem_bytes(ndims, tile.t, tile.s1, tile.s2, tile.s3);
     if (block_threads) *block_threads = thr;
@@ -247,7 +248,7 @@ extern "C" int stencil_tile_occupancy(stencil_kind kind, int ndims, stencil_tile
                                       int* blocks_per_sm) {
     if (!blocks_per_sm || kind_ndims_host(kind) != ndims) return STENCIL_EINVAL;
     int G, thr;
-    const int rc = check_tile(ndims, tile, threads, 227 * 1024, &G, &thr);
+    const int rc = check_tile(ndims, tile, threads, 227 * 1024, &G, &thr, kind);
     if (rc) return rc;
     hex_kernel_t k = get_hex_kernel(ndims, kind, mode, false, true, tile.s2);
     if (!k) return STENCIL_EINVAL;
@@ -512,7 +513,7 @@ extern "C" int stencil_run(stencil_t h, const float* d_in, float* d_out, int64_t
         return cuda_fail(h, cudaGetLastError());
     }
     RunSpec r;
-    int rc = check_tile(h->ndims, tile, threads, h->smem_optin, &r.G, &r.thr);
+    int rc = check_tile(h->ndims, tile, threads, h->smem_optin, &r.G, &r.thr, h->kind);
     if (rc) return rc;
     if (!h->scratch) {
         cudaError_t e = cudaMalloc(&h->scratch, n * sizeof(float));
@@ -531,7 +532,7 @@ extern "C" int stencil_run_planes(stencil_t h, int64_t rows, float* plane0, floa
     if (h->sticky) return h->sticky;
     if (!plane0 || !plane1 || T < 1 || rows < 3) return STENCIL_EINVAL;
     RunSpec r;
-    int rc = check_tile(h->ndims, tile, threads, h->smem_optin, &r.G, &r.thr);
+    int rc = check_tile(h->ndims, tile, threads, h->smem_optin, &r.G, &r.thr, h->kind);
     if (rc) return rc;
     cudaSetDevice(h->device);
     r.planes_mode = 1; r.a = plane0; r.b = plane1;
@@ -647,7 +648,7 @@ extern "C" int stencil_profile(stencil_t h, const float* d_in, float* d_out, int
     if (h->sticky) return h->sticky;
     if (!d_in || !d_out || T < 1) return STENCIL_EINVAL;
     int G, thr;
-    int rc = check_tile(h->ndims, tile, threads, h->smem_optin, &G, &thr);
+    int rc = check_tile(h->ndims, tile, threads, h->smem_optin, &G, &thr, h->kind);
     if (rc) return rc;
     const int64_t n = h->nelem();
     if (!h->scratch) {

@@ -48,7 +48,10 @@ inline int64_t smem_bytes(int ndims, int tT, int tS1, int tS2, int tS3) {
 // Column threads of one x-group: 2D K1 threads own 8 columns (4 pairs of the
 // pair layout), 3D K2 threads 4 consecutive tS3 columns of one tS2 line.
 // Largest block the HHC kernels launch with (their __launch_bounds__).
-inline int max_block_threads(int ndims) { return ndims == 1 ? 256 : ndims == 2 ? 384 : 512; }
+// kind = 0: the largest over the kinds of that dimension (the model's bound).
+inline int max_block_threads(int ndims, int kind = 0) {
+    return ndims == 1 ? 256 : ndims == 2 ? ((kind == 0 || kind == STENCIL_GRADIENT2D) ? 512 : 384) : 512;
+}
 
 inline int column_threads(int ndims, int tS2, int tS3) {
     return ndims == 1 ? 256 : ndims == 2 ? tS2 / 8 : (tS3 / kCols3D) * tS2;

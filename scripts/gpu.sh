@@ -24,7 +24,7 @@ quick)
   c=$1; shift
   for t in "$@"; do
     HHC_BENCH_ALLOW_SHORT=1 timeout 300 python bench.py --config $c --tile ${t%%:*} --threads ${t##*:} --steps ${STEPS:-3} --warmup 3 --no-cpu-baseline --no-e2e > "$OUT/q.json" 2> "$OUT/q.err"
-    python -c "import json;d=json.loads(open('$OUT/q.json').read().splitlines()[-1]);print('$c $t', d['value'], d['ms_per_step'], d['roofline']['frac'])" 2>/dev/null || { echo "$c $t FAILED"; tail -3 "$OUT/q.err"; }
+    python -c "import json;d=json.loads(open('$OUT/q.json').read().splitlines()[-1]);print('$c $t', d['value'], d['ms_per_step'], d['roofline']['frac'])" 2>/dev/null | tee -a $OUT/quick.txt || { echo "$c $t FAILED"; tail -3 "$OUT/q.err"; }
   done;;
 ncu)
   c=$1; k=${KREGEX:-hex}
