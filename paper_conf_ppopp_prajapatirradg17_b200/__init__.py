@@ -25,7 +25,7 @@ KIND_NAMES = {1: "Jacobi-2D 5-point", 2: "Heat-2D 9-point", 3: "Gradient-2D", 4:
               5: "Laplacian-3D 27-point", 6: "Laplacian-2D 5-point"}
 KIND_NDIMS = {1: 2, 2: 2, 3: 2, 4: 3, 5: 3, 6: 2, 7: 1}
 PLAIN, FUSED = 0, 1
-PAPER, EXACT = 0, 1
+PAPER, EXACT, EXACT_G = 0, 1, 2   # EXACT_G: EXACT + x-group rows (DESIGN reading M9)
 
 OK, EINVAL, ETILE, ENOMEM, ECUDA, ENCCL, ENODEV = 0, -1, -2, -3, -4, -5, -6
 

@@ -122,6 +122,7 @@ double talg_exact(int nd, const int64_t* S, int64_t T, const stencil_tile& tl, c
     if (Mtile > hw.m_block_bytes || threads > hhc::max_block_threads(nd)) return std::numeric_limits<double>::infinity();
     const int64_t k = k_exact(Mtile, threads, hw);                                       // Eq. 11
     if (k < 1) return std::numeric_limits<double>::infinity();
+    const int64_t G = nd == 1 ? 1 : std::max<int64_t>(1, threads / hhc::column_threads(nd, (int)tS2, (int)tS3));
     const int64_t P = 2 * tS1 + tT, h = tT / 2;
     const int64_t wA = cdiv(S1 + h, P);                        // reading G2
     const int64_t wB = S1 > tS1 ? cdiv(S1 - tS1, P) : 0;
@@ -154,7 +155,10 @@ double talg_exact(int nd, const int64_t* S, int64_t T, const stencil_tile& tl, c
             else if (tau <= h) reads += 4;
             if (t0 + tau == T || tau == hi - 1) writes += W;
             else if (tau + 1 > h) writes += 4;
-            csum += (double)cdiv(W * inner, hw.n_v);           // Eq. 15 / 27, row by row
+            // reading M9 (geometry 2): the G x-groups split the row, so a level lasts
+            // G*ceil(W/G) rows' worth of the block's vector units
+            const int64_t We = (hw.geometry == 2 && G > 1) ? G * cdiv(W, G) : W;
+            csum += (double)cdiv(We * inner, hw.n_v);          // Eq. 15 / 27, row by row
         }
         double Nsub, mi, mo, extra = 0.0;
         int64_t J = 1;
@@ -242,7 +246,7 @@ extern "C" double model_predict(stencil_kind kind, int ndims, const int64_t* dim
     if (!tile_ok(ndims, tile)) return nan;
     if (hw->n_sm < 1 || hw->n_v < 1 || hw->mtb_sm < 1 || hw->m_sm_bytes < 1 || hw->m_block_bytes < 1) return nan;
     int64_t S[3] = {dims[0] - 2, ndims >= 2 ? dims[1] - 2 : 1, ndims == 3 ? dims[2] - 2 : 1};
-    auto f = hw->geometry == 1 ? talg_exact : talg_paper;
+    auto f = hw->geometry >= 1 ? talg_exact : talg_paper;
     if (hw->n_gpus > 1) return talg_dist(ndims, S, T, tile, *hw, f);
     return f(ndims, S, T, tile, *hw);
 }

@@ -102,7 +102,7 @@ def test_model_predict_matches_oracle_hand_example(lib):
     assert abs(t - 15.96397) < 2e-5
 
 
-@pytest.mark.parametrize("geometry", [hhc.PAPER, hhc.EXACT])
+@pytest.mark.parametrize("geometry", [hhc.PAPER, hhc.EXACT, hhc.EXACT_G])
 def test_model_predict_matches_oracle_random(lib, geometry):
     rnd = random.Random(geometry + 7)
     n = 0
@@ -138,7 +138,7 @@ def test_model_predict_multi_gpu_matches_oracle(lib, overlap):
     for _ in range(200):
         kind = rnd.choice([1, 2, 3, 4, 5])
         nd = hhc.KIND_NDIMS[kind]
-        geometry = rnd.choice([hhc.PAPER, hhc.EXACT])
+        geometry = rnd.choice([hhc.PAPER, hhc.EXACT, hhc.EXACT_G])
         o, c = hw_pair(kind, geometry, rnd, b200=True)
         G = rnd.randint(2, 8)
         o.n_gpus = c.n_gpus = G

@@ -257,3 +257,26 @@ def test_select_tile_small_space():
     assert min(allv)[1] == best and min(allv)[0] == tmin
     assert set(cands) == {tl for t, tl in allv if t <= 1.1 * tmin}
     assert best in cands
+
+
+def test_xgroup_rows_reading_m9():
+    """Reading M9 (EXACT_G): with G x-groups a level costs G*ceil(W/G) rows, so
+    EXACT_G >= EXACT, equal when every row width is a multiple of G (G = 1 or
+    W(tau) divisible), and larger for some tile whose rows do not split evenly."""
+    hw = mo.gtx980(2, mo.EXACT)
+    hw.Mblock, hw.MSM = 227 * 1024, 228 * 1024
+    hwg = mo.gtx980(2, mo.EXACT_G)
+    hwg.Mblock, hwg.MSM = 227 * 1024, 228 * 1024
+    S, T = (2000, 1500), 64
+    larger = 0
+    for tile, thr in [((8, 4, 64, 0), 32), ((8, 4, 64, 0), 8), ((16, 6, 128, 0), 64), ((4, 2, 32, 0), 12)]:
+        hw.threads = hwg.threads = thr
+        te, tg = mo.talg(2, S, T, tile, hw), mo.talg(2, S, T, tile, hwg)
+        G = thr // (tile[2] // 8)
+        widths = {mo.row_width(t, tile[1], tile[0]) for t in range(tile[0])}
+        if G == 1 or all(w % G == 0 for w in widths):
+            assert te == tg
+        else:
+            assert tg >= te
+            larger += tg > te
+    assert larger >= 1
