@@ -47,6 +47,9 @@ CONFIGS = {
     # SURVEY §8(f) f3 (not a BASELINE.json config): the wavefront-parallel schedule
     "W1": dict(kind=7, dims=((1 << 22) + 2,), T=1024, tile=(4, 8192), threads=256, schedule="wavefront",
                desc="Jacobi-1D 3-point fp32, 2^22 interior points, T=1024, wavefront schedule (extension f3)"),
+    # SURVEY §8(f) f4 (not a BASELINE.json config): a higher-order (radius-2) stencil under HHC
+    "X2": dict(kind=8, dims=(1 << 26,), T=1024, tile=(64, 2048), threads=256,
+               desc="Binomial-1D radius-2 5-point fp32, 2^26 points, T=1024 (extension f4)"),
 }
 DEFAULT_CONFIG = "C3"
 
@@ -55,7 +58,7 @@ DEFAULT_CONFIG = "C3"
 # |N|-1 FFMA of the canonical fused expression).  Gradient-2D: counted in the
 # kernel's SASS (FP32-pipe lane ops of the IEEE sqrt and division sequences
 # included, MUFU excluded), scripts/count_fp32.py -> profiles/r02/n_fp32_gradient.txt.
-N_FP32 = {1: 5, 2: 9, 3: 24.5, 4: 7, 5: 27, 6: 5, 7: 3}
+N_FP32 = {1: 5, 2: 9, 3: 24.5, 4: 7, 5: 27, 6: 5, 7: 3, 8: 5, 9: 7, 10: 9}
 N_FP32_SOURCE = {3: "SASS count of the Gradient-2D row step (profiles/r02/n_fp32_gradient.txt)"}
 
 METRIC = "GStencil-updates/s"
@@ -154,6 +157,12 @@ def ncu_traffic(cfg: str):
     return None
 
 
+def hhc_updates(dims, T, kind):
+    """Interior updates T * prod(S_d - 2R), R the kind's ring width (1; 2-4 for f4)."""
+    R = {8: 2, 9: 3, 10: 4}.get(int(kind), 1)
+    return int(T) * math.prod(int(d) - 2 * R for d in dims)
+
+
 def cpu_oracle_sample(cfg: dict, seconds: float = 10.0, nthreads: int = 0):
     """The oracle as it stands (plain mode, all host cores) on a bounded sample
     of the workload: the full grid for T_s < T steps, T_s sized to ~`seconds`."""
@@ -161,7 +170,7 @@ def cpu_oracle_sample(cfg: dict, seconds: float = 10.0, nthreads: int = 0):
     from synth import CONFIG_SEEDS, field
     name = [k for k, v in CONFIGS.items() if v is cfg][0]
     a = field(CONFIG_SEEDS[name], cfg["dims"])
-    n_int = math.prod(d - 2 for d in cfg["dims"])
+    n_int = hhc_updates(cfg["dims"], 1, cfg["kind"])
     oracle.run(cfg["kind"], a, 1, oracle.PLAIN, nthreads=nthreads)        # warm (threads, first touch)
     t0 = time.perf_counter()
     oracle.run(cfg["kind"], a, 2, oracle.PLAIN, nthreads=nthreads)
@@ -189,7 +198,7 @@ def run_reference(args, cfg, cfgname):
     if rank != 0:
         return 0
     a = field(CONFIG_SEEDS[cfgname], cfg["dims"])
-    n_int = math.prod(d - 2 for d in cfg["dims"])
+    n_int = hhc_updates(cfg["dims"], 1, cfg["kind"])
     t0 = time.perf_counter()
     oracle.run(cfg["kind"], a, 1, oracle.PLAIN)
     one = max(time.perf_counter() - t0, 1e-4)
@@ -257,7 +266,7 @@ def bench_single(args, cfg, cfgname):
     threads = cfg["threads"] if args.threads is None else args.threads
     mode = hhc.FUSED if args.mode == "fused" else hhc.PLAIN
     dims, T, kind = cfg["dims"], cfg["T"], cfg["kind"]
-    n_upd = hhc.updates(dims, T)
+    n_upd = hhc.updates(dims, T, kind)
 
     host = field(CONFIG_SEEDS[cfgname], dims)
     h_in = torch.from_numpy(host).pin_memory()

@@ -46,8 +46,16 @@ typedef enum {
     STENCIL_HEAT3D_7PT = 4,        /* centre + 6 faces, 1/4, 1/8                            */
     STENCIL_LAPLACIAN3D_27PT = 5,  /* 3x3x3 box, 1/2, 7/128, 3/256, 1/256                   */
     STENCIL_LAPLACIAN2D_5PT = 6,   /* centre + 4 faces, 1/2, 1/8                            */
-    STENCIL_JACOBI1D_3PT = 7       /* 1D: x-1, x, x+1, weights fp32(1/3) (the
+    STENCIL_JACOBI1D_3PT = 7,      /* 1D: x-1, x, x+1, weights fp32(1/3) (the
                                       paper's Section 4.1 derivation)           */
+    /* SURVEY §8(f) f4, higher-order stencils ("Generality": the hexagon
+     * slopes and footprints change by constant factors): 1D radius-r binomial
+     * smoothers, offsets -r..r, weights C(2r, r+d) / 4^r.  For these kinds the fixed
+     * boundary ring is r cells wide (interior [r, S1-1-r]), hexagon rows widen by 2r
+     * per level (pitch 2 tS1 + r tT), footprints/facets are 2r rows per side. */
+    STENCIL_BINOM1D_R2 = 8,        /* 5-point,  1 4 6 4 1 / 16                              */
+    STENCIL_BINOM1D_R3 = 9,        /* 7-point,  1 6 15 20 15 6 1 / 64                       */
+    STENCIL_BINOM1D_R4 = 10        /* 9-point,  1 8 28 56 70 56 28 8 1 / 256                */
 } stencil_kind;
 
 typedef enum {

@@ -28,7 +28,9 @@ _LIB = os.path.join(_HERE, "liboracle.so")
 
 JACOBI2D_5PT, HEAT2D_9PT, GRADIENT2D, HEAT3D_7PT, LAPLACIAN3D_27PT, LAPLACIAN2D_5PT = 1, 2, 3, 4, 5, 6
 JACOBI1D_3PT = 7
-KIND_NDIMS = {1: 2, 2: 2, 3: 2, 4: 3, 5: 3, 6: 2, 7: 1}
+BINOM1D_R2, BINOM1D_R3, BINOM1D_R4 = 8, 9, 10      # radius-r 1D binomial smoothers
+KIND_NDIMS = {1: 2, 2: 2, 3: 2, 4: 3, 5: 3, 6: 2, 7: 1, 8: 1, 9: 1, 10: 1}
+KIND_RADIUS = {8: 2, 9: 3, 10: 4}
 PLAIN, FUSED = 0, 1
 
 CFLAGS = ["-O2", "-ffp-contract=off", "-fno-fast-math", "-fopenmp", "-shared", "-fPIC"]

@@ -14,6 +14,11 @@ x0 - m(tau) <= x < x0 + tS + m(tau), with m(tau) = min(tau, tT - tau).
 Lattice (reading G2): phase A corners at (1 + k*tT, 1 + j*P), phase B corners
 at (1 - tT/2 + k*tT, 1 + tS + tT/2 + j*P); the row index of a tile is
 m = (t0 - 1) / (tT/2), even for A, odd for B.
+
+Radius R (reading F4; "the slopes of the
+hexagons change by constant factors"): m(tau) = R min(tau, tT - tau), pitch
+P = 2tS + R tT, phase B corners at x = 1 + tS + R tT/2 + j*P, and a point
+depends on (t-1, x-R .. x+R).  R = 1 is the paper's first-order case.
 """
 from __future__ import annotations
 
@@ -24,10 +29,10 @@ def hexagon_rows(tS: int, tT: int):
     return [(tau, -min(tau, tT - tau), tS + min(tau, tT - tau)) for tau in range(tT)]
 
 
-def tile_of(t: int, x: int, tS: int, tT: int):
+def tile_of(t: int, x: int, tS: int, tT: int, R: int = 1):
     """Return the unique (m, j) whose hexagon contains (t, x); raises if the
     point is covered zero or several times."""
-    P = 2 * tS + tT
+    P = 2 * tS + R * tT
     h = tT // 2
     hits = []
     # candidate rows: the point's level lies in [t0, t0 + tT)
@@ -36,8 +41,8 @@ def tile_of(t: int, x: int, tS: int, tT: int):
         tau = t - t0
         if not (0 <= tau < tT):
             continue
-        base = 1 if m % 2 == 0 else 1 + tS + h
-        mm = min(tau, tT - tau)
+        base = 1 if m % 2 == 0 else 1 + tS + R * h
+        mm = R * min(tau, tT - tau)
         # x0 - mm <= x < x0 + tS + mm with x0 = base + j*P
         for j in range((x - base - tS - mm) // P - 1, (x - base + mm) // P + 2):
             x0 = base + j * P
@@ -48,17 +53,17 @@ def tile_of(t: int, x: int, tS: int, tT: int):
     return hits[0]
 
 
-def enumerate_tiling(S1: int, T: int, tS: int, tT: int):
+def enumerate_tiling(S1: int, T: int, tS: int, tT: int, R: int = 1):
     """Map every point of [1,T] x [1,S1] to its tile.  Returns
     tiles: {(m, j): set of (t, x)}."""
     tiles = defaultdict(set)
     for t in range(1, T + 1):
         for x in range(1, S1 + 1):
-            tiles[tile_of(t, x, tS, tT)].add((t, x))
+            tiles[tile_of(t, x, tS, tT, R)].add((t, x))
     return tiles
 
 
-def analyse(S1: int, T: int, tS: int, tT: int):
+def analyse(S1: int, T: int, tS: int, tT: int, R: int = 1):
     """Brute-force statistics of the tiling:
     rows: sorted list of non-empty row indices (= kernel launches, Nw);
     w: {m: number of non-empty tiles in row m};
@@ -68,7 +73,7 @@ def analyse(S1: int, T: int, tS: int, tT: int):
     and checks the schedule: every dependence (t-1, x+d) of a point is either
     level 0 / the ring, in the same tile at an earlier level, or in a tile of
     an EARLIER row (never the same row)."""
-    tiles = enumerate_tiling(S1, T, tS, tT)
+    tiles = enumerate_tiling(S1, T, tS, tT, R)
     owner = {}
     for key, pts in tiles.items():
         for p in pts:
@@ -82,7 +87,7 @@ def analyse(S1: int, T: int, tS: int, tT: int):
     for key, pts in tiles.items():
         need = set()
         for (t, x) in pts:
-            for d in (-1, 0, 1):
+            for d in range(-R, R + 1):
                 q = (t - 1, x + d)
                 if q[0] == 0 or q[1] < 1 or q[1] > S1:
                     continue            # initial value or ring: read from the input
@@ -98,7 +103,7 @@ def analyse(S1: int, T: int, tS: int, tT: int):
             if t == T:
                 wr += 1
                 continue
-            for d in (-1, 0, 1):
+            for d in range(-R, R + 1):
                 q = (t + 1, x + d)
                 if 1 <= q[1] <= S1 and owner[q] != key:
                     wr += 1

@@ -30,8 +30,12 @@
 
 /* Stencil kinds (numbering is part of the C ABI contract in include/hhc.h,
  * re-declared here on purpose: the oracle includes nothing from the product). */
-enum { O_JACOBI2D_5PT = 1, O_HEAT2D_9PT = 2, O_GRADIENT2D = 3,
-       O_HEAT3D_7PT = 4, O_LAPLACIAN3D_27PT = 5, O_LAPLACIAN2D_5PT = 6, O_JACOBI1D_3PT = 7 };
+enum { O_JACOBI1D_3PT = 7,
+       O_JACOBI2D_5PT = 1, O_HEAT2D_9PT = 2, O_GRADIENT2D = 3,
+       O_HEAT3D_7PT = 4, O_LAPLACIAN3D_27PT = 5, O_LAPLACIAN2D_5PT = 6,
+       /* SURVEY §8(f) f4, higher-order stencils ("Generality"):
+        * 1D radius-r binomial smoothers, r = 2, 3, 4 */
+       O_BINOM1D_R2 = 8, O_BINOM1D_R3 = 9, O_BINOM1D_R4 = 10 };
 enum { O_MODE_PLAIN = 0, O_MODE_FUSED = 1 };
 
 typedef struct {
@@ -49,9 +53,14 @@ static int o_kind_ndims(int kind) {
     switch (kind) {
     case O_JACOBI2D_5PT: case O_HEAT2D_9PT: case O_GRADIENT2D: case O_LAPLACIAN2D_5PT: return 2;
     case O_HEAT3D_7PT: case O_LAPLACIAN3D_27PT: return 3;
-    case O_JACOBI1D_3PT: return 1;
+    case O_JACOBI1D_3PT: case O_BINOM1D_R2: case O_BINOM1D_R3: case O_BINOM1D_R4: return 1;
     default: return 0;
     }
+}
+
+/* Radius of the neighbourhood: 1, or r for the f4 kinds (offsets -r..r). */
+static int o_kind_radius(int kind) {
+    return kind == O_BINOM1D_R2 ? 2 : kind == O_BINOM1D_R3 ? 3 : kind == O_BINOM1D_R4 ? 4 : 1;
 }
 
 /* Is offset (number of non-zero components = nz) in N_kind? */
@@ -94,6 +103,18 @@ static int o_build(int kind, const float* coeffs, int ncoeffs, o_stencil* s) {
         return 0;
     }
     int D = s->ndims;
+    int r = o_kind_radius(kind);
+    if (r > 1) {
+        /* binomial weights C(2r, k) / 4^r on the offsets -r..r (dyadic, positive, sum 1) */
+        double c = 1.0, den = 1.0;
+        for (int k = 0; k < 2 * r; ++k) den *= 2.0;
+        for (int k = 0; k <= 2 * r; ++k) {
+            s->off[s->n][0] = k - r; s->off[s->n][1] = 0; s->off[s->n][2] = 0;
+            s->w[s->n] = (float)(c / den);
+            s->n++;
+            c = c * (double)(2 * r - k) / (double)(k + 1);
+        }
+    } else {
     int lo3 = (D == 3) ? -1 : 0, hi3 = (D == 3) ? 1 : 0;
     int lo2 = (D >= 2) ? -1 : 0, hi2 = (D >= 2) ? 1 : 0;
     for (int d1 = -1; d1 <= 1; ++d1)
@@ -105,6 +126,7 @@ static int o_build(int kind, const float* coeffs, int ncoeffs, o_stencil* s) {
                 s->w[s->n] = o_default_weight(kind, nz);
                 s->n++;
             }
+    }
     if (coeffs) {
         if (ncoeffs != s->n && ncoeffs != s->n + 1) return -1;
         for (int j = 0; j < s->n; ++j) s->w[j] = coeffs[j];
@@ -157,7 +179,7 @@ int oracle_run(int kind, int ndims, const int64_t* dims, const float* coeffs, in
     if (ndims != s.ndims || T < 0 || !in || !out) return -1;
     if (mode != O_MODE_PLAIN && mode != O_MODE_FUSED) return -1;
     int64_t S1 = dims[0], S2 = (ndims >= 2) ? dims[1] : 1, S3 = (ndims == 3) ? dims[2] : 1;
-    if (S1 < 3 || (ndims >= 2 && S2 < 3) || (ndims == 3 && S3 < 3)) return -1;
+    if (S1 < 2 * o_kind_radius(kind) + 1 || (ndims >= 2 && S2 < 3) || (ndims == 3 && S3 < 3)) return -1;
     int64_t n = S1 * S2 * S3;
     int64_t stride[3] = { S2 * S3, S3, 1 };
     if (ndims == 2) { stride[0] = S2; stride[1] = 1; stride[2] = 0; }
@@ -173,8 +195,10 @@ int oracle_run(int kind, int ndims, const int64_t* dims, const float* coeffs, in
         const float* src = plane[(t - 1) & 1];
         float* dst = plane[t & 1];
         if (ndims == 1) {
+            /* the fixed ring is r cells wide for a radius-r neighbourhood (reading R2) */
+            const int64_t r = o_kind_radius(kind);
             #pragma omp parallel for num_threads(nt) schedule(static)
-            for (int64_t x = 1; x < S1 - 1; ++x) dst[x] = o_point_linear(&s, src, x, stride, mode);
+            for (int64_t x = r; x < S1 - r; ++x) dst[x] = o_point_linear(&s, src, x, stride, mode);
         } else if (ndims == 2) {
             #pragma omp parallel for num_threads(nt) schedule(static)
             for (int64_t x = 1; x < S1 - 1; ++x)

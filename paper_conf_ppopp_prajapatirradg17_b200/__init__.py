@@ -21,9 +21,12 @@ LIB_PATH = os.path.join(_HERE, "libhhc.so")
 # stencil_kind (include/hhc.h)
 JACOBI2D_5PT, HEAT2D_9PT, GRADIENT2D, HEAT3D_7PT, LAPLACIAN3D_27PT, LAPLACIAN2D_5PT = 1, 2, 3, 4, 5, 6
 JACOBI1D_3PT = 7          # the paper's 1D derivation case
+BINOM1D_R2, BINOM1D_R3, BINOM1D_R4 = 8, 9, 10   # radius-r 1D binomial smoothers
 KIND_NAMES = {1: "Jacobi-2D 5-point", 2: "Heat-2D 9-point", 3: "Gradient-2D", 4: "Heat-3D 7-point",
-              5: "Laplacian-3D 27-point", 6: "Laplacian-2D 5-point"}
-KIND_NDIMS = {1: 2, 2: 2, 3: 2, 4: 3, 5: 3, 6: 2, 7: 1}
+              5: "Laplacian-3D 27-point", 6: "Laplacian-2D 5-point", 7: "Jacobi-1D 3-point",
+              8: "Binomial-1D radius 2", 9: "Binomial-1D radius 3", 10: "Binomial-1D radius 4"}
+KIND_NDIMS = {1: 2, 2: 2, 3: 2, 4: 3, 5: 3, 6: 2, 7: 1, 8: 1, 9: 1, 10: 1}
+KIND_RADIUS = {8: 2, 9: 3, 10: 4}
 PLAIN, FUSED = 0, 1
 PAPER, EXACT, EXACT_G = 0, 1, 2   # EXACT_G: EXACT + x-group rows (DESIGN reading M9)
 
@@ -366,9 +369,11 @@ def stencil_microbench(which: int, kind: int = HEAT2D_9PT, dims=(3, 3), T: int =
     return v.value
 
 
-def updates(dims, T: int) -> int:
-    """Interior stencil updates of a run: T * prod(S_d - 2)."""
-    return int(T) * math.prod(int(x) - 2 for x in dims)
+def updates(dims, T: int, kind: int = 0) -> int:
+    """Interior stencil updates of a run: T * prod(S_d - 2R) (ring width R = 1,
+    2-4 for the f4 kinds)."""
+    R = KIND_RADIUS.get(int(kind), 1)
+    return int(T) * math.prod(int(x) - 2 * R for x in dims)
 
 
 EXPORTED_SYMBOLS = ["stencil_create", "stencil_destroy", "stencil_run", "stencil_run_host",

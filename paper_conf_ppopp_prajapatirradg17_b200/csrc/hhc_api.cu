@@ -20,7 +20,7 @@ int kind_ndims_host(int kind) {
     case STENCIL_JACOBI2D_5PT: case STENCIL_HEAT2D_9PT: case STENCIL_GRADIENT2D:
     case STENCIL_LAPLACIAN2D_5PT: return 2;
     case STENCIL_HEAT3D_7PT: case STENCIL_LAPLACIAN3D_27PT: return 3;
-    case STENCIL_JACOBI1D_3PT: return 1;
+    case STENCIL_JACOBI1D_3PT: case STENCIL_BINOM1D_R2: case STENCIL_BINOM1D_R3: case STENCIL_BINOM1D_R4: return 1;
     default: return 0;
     }
 }
@@ -96,6 +96,7 @@ struct stencil_s {
     int occ = 1;
     int envJ = 0;               // HHC_J read once at create (experiments; 0 = library rule)
     int maxJ = 0;               // > 0: cap on the 3D blocks per slab (1 = never wait on flags)
+    int R = 1;                  // stencil radius = fixed-ring width (f4 kinds: 2-4)
 
     int64_t nelem() const { return dims[0] * dims[1] * dims[2]; }
 };
@@ -151,6 +152,27 @@ extern "C" int stencil_create(stencil_kind kind, int ndims, const int64_t* dims,
             h->kappa = coeffs[0];
             h->defw = h->kappa == 0.125f;
         }
+    } else if (kind_radius(kind) > 1) {
+        // f4: binomial C(2R, j) / 4^R on the offsets -R..R (reading R1)
+        const int R = kind_radius(kind);
+        h->R = R;
+        h->npts = 2 * R + 1;
+        double c = 1.0;
+        for (int j = 0; j <= 2 * R; ++j) {
+            h->w[j] = (float)(c / (double)(1 << (2 * R)));
+            c = c * (double)(2 * R - j) / (double)(j + 1);
+        }
+        for (int d = 0; d < ndims; ++d)
+            if (dims[d] < 2 * R + 1) { delete h; return STENCIL_EINVAL; }
+        if (coeffs) {
+            const int n = h->npts;
+            if (ncoeffs != n && ncoeffs != n + 1) { delete h; return STENCIL_EINVAL; }
+            for (int j = 0; j < n; ++j) {
+                if (coeffs[j] != h->w[j] || std::signbit(coeffs[j]) != std::signbit(h->w[j])) h->defw = false;
+                h->w[j] = coeffs[j];
+            }
+            if (ncoeffs == n + 1 && coeffs[n] != 0.0f) { h->has_c = true; h->c = coeffs[n]; h->defw = false; }
+        }
     } else {
         int n = 0;
         for (int d1 = -1; d1 <= 1; ++d1)
@@ -197,7 +219,7 @@ static int check_tile(int ndims, stencil_tile t, int threads, int smem_limit, in
     if (ndims == 1) {
         if (t.t > 1024 || t.s1 > 65536) return STENCIL_ETILE;
         if (threads != 0 && threads != 256) return STENCIL_EINVAL;
-        const int64_t sm = smem_bytes(1, t.t, t.s1, 0, 0);
+        const int64_t sm = smem_bytes(1, t.t, t.s1, 0, 0, kind_radius(kind));
         if (sm > smem_limit) return STENCIL_ETILE;
         *G_out = 1;
         *thr_out = 256;
@@ -232,7 +254,7 @@ extern "C" int stencil_tile_resources(stencil_kind kind, int ndims, stencil_tile
     int G, thr;
     const int rc = check_tile(ndims, tile, threads, 227 * 1024, &G, &thr, kind);
     if (rc) return rc;
-    if (smem) *smem = smem_bytes(ndims, tile.t, tile.s1, tile.s2, tile.s3);
+    if (smem) *smem = smem_bytes(ndims, tile.t, tile.s1, tile.s2, tile.s3, kind_radius(kind));
     if (block_threads) *block_threads = thr;
     if (regs) {
         // Eq. 11's register bound (reading M4): the kernel the library launches for this
@@ -252,7 +274,7 @@ extern "C" int stencil_tile_occupancy(stencil_kind kind, int ndims, stencil_tile
     if (rc) return rc;
     hex_kernel_t k = get_hex_kernel(ndims, kind, mode, false, true, tile.s2);
     if (!k) return STENCIL_EINVAL;
-    const int64_t smem = smem_bytes(ndims, tile.t, tile.s1, tile.s2, tile.s3);
+    const int64_t smem = smem_bytes(ndims, tile.t, tile.s1, tile.s2, tile.s3, kind_radius(kind));
     cudaError_t e = cudaFuncSetAttribute((const void*)k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, (const void*)k, thr, (size_t)smem);
     if (e != cudaSuccess) {
@@ -263,13 +285,16 @@ extern "C" int stencil_tile_occupancy(stencil_kind kind, int ndims, stencil_tile
 }
 
 // ---- planning (a1, a3): rows m = -1 .. Nw-2 (reading G2)
-static void plan_rows(int ndims, const int64_t* dims, int64_t T, stencil_tile t, std::vector<RowPlan>& rows) {
+static void plan_rows(int ndims, const int64_t* dims, int64_t T, stencil_tile t, std::vector<RowPlan>& rows,
+                      int R = 1) {
+    // radius R (f4): ring of width R, interior [R, S1-1-R], rows widen by R per
+    // level side, pitch P = 2 tS1 + R tT, phase B at x0 + tS1 + R tT/2
     rows.clear();
-    const int64_t S1i = dims[0] - 2;
+    const int64_t S1i = dims[0] - 2 * R;
     const int h = t.t / 2;
-    const int P = 2 * t.s1 + t.t;
+    const int P = 2 * t.s1 + R * t.t;
     const int64_t Nw = cdiv(2 * T, t.t) + 1;
-    const int64_t wA = cdiv(S1i + h, P);
+    const int64_t wA = cdiv(S1i + (int64_t)R * h, P);
     const int64_t wB = S1i > t.s1 ? cdiv(S1i - t.s1, P) : 0;
     for (int64_t m = -1; m <= Nw - 2; ++m) {
         RowPlan r;
@@ -278,7 +303,7 @@ static void plan_rows(int ndims, const int64_t* dims, int64_t T, stencil_tile t,
         r.tau_lo = (int)std::max<int64_t>(0, 1 - r.t0);
         r.tau_hi = (int)std::min<int64_t>(t.t, T - r.t0 + 1);
         const bool A = (m % 2 == 0);
-        r.xbase = A ? 1 : 1 + t.s1 + h;
+        r.xbase = A ? R : R + t.s1 + (int64_t)R * h;
         r.w = (int)(A ? wA : wB);
         const int nlev = r.tau_hi - r.tau_lo;
         if (ndims == 1) {
@@ -330,7 +355,7 @@ static int choose_J(stencil_t h, const RowPlan& r) {
 static int prepare_rows(stencil_t h, const int64_t* dims, int64_t T, stencil_tile tile, int thr) {
     hex_kernel_t k = get_hex_kernel(h->ndims, h->kind, h->mode, h->has_c, h->defw, tile.s2);
     if (!k) return STENCIL_EINVAL;
-    const int64_t smem = smem_bytes(h->ndims, tile.t, tile.s1, tile.s2, tile.s3);
+    const int64_t smem = smem_bytes(h->ndims, tile.t, tile.s1, tile.s2, tile.s3, h->R);
     cudaError_t e = cudaFuncSetAttribute((const void*)k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return cuda_fail(h, e);
     if (h->ndims != 3) return STENCIL_OK;
@@ -339,7 +364,7 @@ static int prepare_rows(stencil_t h, const int64_t* dims, int64_t T, stencil_til
     if (e != cudaSuccess) return cuda_fail(h, e);
     h->occ = std::max(occ, 1);
     std::vector<RowPlan> rows;
-    plan_rows(h->ndims, dims, T, tile, rows);
+    plan_rows(h->ndims, dims, T, tile, rows, h->R);
     int64_t need = 0;
     for (auto& r : rows) {
         const int J = choose_J(h, r);
@@ -366,10 +391,10 @@ static int enqueue_rows(stencil_t h, const int64_t* dims, const float* ring, flo
                         int64_t T, stencil_tile tile, int G, int thr, cudaStream_t s, int64_t* launches,
                         std::vector<cudaEvent_t>* evs = nullptr) {
     std::vector<RowPlan> rows;
-    plan_rows(h->ndims, dims, T, tile, rows);
+    plan_rows(h->ndims, dims, T, tile, rows, h->R);
     hex_kernel_t k = get_hex_kernel(h->ndims, h->kind, h->mode, h->has_c, h->defw, tile.s2);
     if (!k) return STENCIL_EINVAL;
-    const int64_t smem = smem_bytes(h->ndims, tile.t, tile.s1, tile.s2, tile.s3);
+    const int64_t smem = smem_bytes(h->ndims, tile.t, tile.s1, tile.s2, tile.s3, h->R);
     int64_t nl = 0;
     cudaError_t e;
     // 3D: thread blocks per slab J (pipelined along S2, flags in global memory);
@@ -396,7 +421,8 @@ static int enqueue_rows(stencil_t h, const int64_t* dims, const float* ring, flo
     p.T = T;
     p.tT = tile.t; p.tS1 = tile.s1; p.tS2 = tile.s2; p.tS3 = h->ndims == 3 ? tile.s3 : 0;
     p.G = G;
-    p.P = 2 * tile.s1 + tile.t;
+    p.P = 2 * tile.s1 + h->R * tile.t;
+    p.R = h->R;
     for (int j = 0; j < kMaxPts; ++j) p.w[j] = h->w[j];
     p.c = h->c;
     p.kappa = h->kappa;
@@ -437,11 +463,11 @@ static int enqueue_spec(stencil_t h, const RunSpec& r, cudaStream_t s, int64_t* 
         plane[1 - (r.T & 1)] = h->scratch;
         // a2: level 0 in plane 0, the fixed ring in plane 1 (readings R2/R3)
         launch_copy_full(r.a, plane[0], n, s); ++nl;
-        launch_copy_ring(r.a, plane[1], r.dims[0], r.dims[1], r.dims[2], s); ++nl;
+        launch_copy_ring(r.a, plane[1], r.dims[0], r.dims[1], r.dims[2], s, h->R); ++nl;
         rc = enqueue_rows(h, r.dims, r.a, plane[0], plane[1], r.T, r.tile, r.G, r.thr, s, &nrows, nullptr);
     } else {
         float* p0 = const_cast<float*>(r.a);
-        launch_copy_ring(p0, r.b, r.dims[0], r.dims[1], r.dims[2], s); ++nl;
+        launch_copy_ring(p0, r.b, r.dims[0], r.dims[1], r.dims[2], s, h->R); ++nl;
         rc = enqueue_rows(h, r.dims, p0, p0, r.b, r.T, r.tile, r.G, r.thr, s, &nrows, nullptr);
     }
     *launches = nl + nrows;
@@ -660,7 +686,7 @@ extern "C" int stencil_profile(stencil_t h, const float* d_in, float* d_out, int
     plane[T & 1] = d_out;
     plane[1 - (T & 1)] = h->scratch;
     launch_copy_full(d_in, plane[0], n, s);
-    launch_copy_ring(d_in, plane[1], h->dims[0], h->dims[1], h->dims[2], s);
+    launch_copy_ring(d_in, plane[1], h->dims[0], h->dims[1], h->dims[2], s, h->R);
     rc = prepare_rows(h, h->dims, T, tile, thr);
     if (rc) return rc;
     std::vector<cudaEvent_t> evs;
@@ -689,6 +715,8 @@ namespace hhc {
 void set_compute_only(stencil_t h, int on) { if (h) h->compute_only = on; }
 
 void set_last_launches(stencil_t h, int64_t n) { if (h) h->last_launches = n; }
+
+int handle_radius(stencil_t h) { return h ? h->R : 1; }
 
 void handle_info(stencil_t h, int* kind, int* ndims, int64_t* dims, int* device) {
     *kind = h->kind;

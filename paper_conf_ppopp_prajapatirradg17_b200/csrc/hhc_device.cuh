@@ -164,20 +164,21 @@ __device__ __forceinline__ void ld6(const float* base, float (&r)[6]) {
     r[0] = h.x; r[1] = h.y; r[2] = m.x; r[3] = m.y; r[4] = m.z; r[5] = m.w;
 }
 
-// Clipped row [l, r) of local level lev (reading G1); empty (l == r) outside [0, nlev).
+// Clipped row [l, r) of local level lev (reading G1; radius R: slopes and the
+// fixed ring scale by R); empty (l == r) outside [0, nlev).
 __device__ __forceinline__ void hex_row(const HexParams& p, int64_t x0, int nlev, int lev,
                                         int64_t& l, int64_t& r) {
     if (lev < 0 || lev >= nlev) { l = r = 0; return; }
     const int tau = p.tau_lo + lev;
-    const int mm = min(tau, p.tT - tau);
-    l = max(x0 - mm, (int64_t)1);
-    r = min(x0 + p.tS1 + mm, p.S1 - 1);
+    const int mm = p.R * min(tau, p.tT - tau);
+    l = max(x0 - mm, (int64_t)p.R);
+    r = min(x0 + p.tS1 + mm, p.S1 - p.R);
     if (r < l) r = l;
 }
 
 // Footprint of local level lev (values of level lev-1 the block does not hold):
-// F = (row(lev) +- 1) \ row(lev-1), as two intervals, plus the interval of
-// row(lev-1) positions inside row(lev)+-1 ("inner").  first = no usable row(lev-1).
+// F = (row(lev) +- R) \ row(lev-1), as two intervals, plus the interval of
+// row(lev-1) positions inside row(lev)+-R ("inner").  first = no usable row(lev-1).
 struct Foot { int64_t A0, A1, f1a, f1b, f2a, f2b, ia, ib; bool first, empty; };
 
 __device__ __forceinline__ Foot footprint(const HexParams& p, int64_t x0, int nlev, int lev) {
@@ -186,7 +187,7 @@ __device__ __forceinline__ Foot footprint(const HexParams& p, int64_t x0, int nl
     hex_row(p, x0, nlev, lev, rl, rr);
     hex_row(p, x0, nlev, lev - 1, pl, pr);
     f.empty = rl >= rr;
-    f.A0 = rl - 1; f.A1 = rr + 1;
+    f.A0 = rl - p.R; f.A1 = rr + p.R;
     f.first = (lev == 0) || (pl >= pr);
     if (f.first) {
         f.f1a = f.A0; f.f1b = f.A1; f.f2a = f.f2b = f.A1; f.ia = f.ib = f.A1;
@@ -198,14 +199,6 @@ __device__ __forceinline__ Foot footprint(const HexParams& p, int64_t x0, int nl
         if (f.ib < f.ia) f.ib = f.ia;
     }
     return f;
-}
-
-// Facet rule (reading G3): (lev, x) is written iff some reader (lev+1, x'),
-// |x'-x| <= 1, x' interior, is not computed by this block, or lev is level T.
-__device__ __forceinline__ bool is_facet(int64_t x, int64_t nl, int64_t nr, int64_t S1, bool final_level) {
-    if (final_level || nl >= nr) return true;
-    const int64_t lo = max(x - 1, (int64_t)1), hi = min(x + 1, S1 - 2);
-    return !(lo >= nl && hi < nr);
 }
 
 // Asynchronous 4-byte global -> shared copy (LDGSTS); the footprint rows are
@@ -235,13 +228,14 @@ __device__ __forceinline__ void cp_async_f4(float* dst, const float* src) {
 }
 
 // Non-facet interval [lo, hi) of smem rows at one level (reading G3): rows whose
-// every reader at the next level lies inside this block.  Empty -> write all.
+// every reader at the next level, x' in [x-R, x+R] within the interior
+// [R, S1-1-R], lies inside this block's next row [nl, nr).  Empty -> write all.
 __device__ __forceinline__ void facet_gap(int64_t nl, int64_t nr, int64_t S1, bool final_level, int64_t xs,
-                                          int NX, int& lo, int& hi) {
+                                          int NX, int R, int& lo, int& hi) {
     lo = hi = 0;
     if (final_level || nl >= nr) return;
-    const int64_t xl = nl <= 1 ? (int64_t)-4 + xs : nl + 1;        // max(x-1,1) >= nl
-    const int64_t xh = nr >= S1 - 1 ? xs + NX + 4 : nr - 1;        // min(x+1,S1-2) < nr
+    const int64_t xl = nl <= R ? (int64_t)-4 + xs : nl + R;         // max(x-R,R) >= nl
+    const int64_t xh = nr >= S1 - R ? xs + NX + 4 : nr - R;        // min(x+R,S1-1-R) < nr
     if (xl >= xh) return;
     lo = (int)max(xl - xs, (int64_t)-2);
     hi = (int)min(xh - xs, (int64_t)NX + 2);
@@ -253,7 +247,7 @@ __device__ __forceinline__ void facet_gap(int64_t nl, int64_t nr, int64_t S1, bo
 //  8, 9 the row [rl, rr); 10, 11 the non-facet gap [lo, hi); 12 rows per x-group.
 constexpr int kGeo = 16;
 __device__ __forceinline__ void build_geo(const HexParams& p, int64_t x0, int64_t xs, int nlev, int* geo) {
-    const int NX = p.tS1 + p.tT + 2;
+    const int NX = p.tS1 + p.R * p.tT + 2 * p.R;
     const int64_t tb = p.t0 + p.tau_lo;
     for (int lev = threadIdx.x; lev < nlev; lev += blockDim.x) {
         const Foot f = footprint(p, x0, nlev, lev);
@@ -267,7 +261,7 @@ __device__ __forceinline__ void build_geo(const HexParams& p, int64_t x0, int64_
         hex_row(p, x0, nlev, lev + 1, nl, nr);
         g[8] = (int)(rl - xs); g[9] = (int)(rr - xs);
         int lo, hi;
-        facet_gap(nl, nr, p.S1, tb + lev == p.T, xs, NX, lo, hi);
+        facet_gap(nl, nr, p.S1, tb + lev == p.T, xs, NX, p.R, lo, hi);
         g[10] = lo; g[11] = hi;
         g[12] = (int)((rr - rl + p.G - 1) / p.G);
     }

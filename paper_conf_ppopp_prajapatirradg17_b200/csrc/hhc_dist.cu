@@ -120,6 +120,7 @@ struct Rank {
         int kind, nd, dev;
         int64_t dims[3];
         hhc::handle_info(h, &kind, &nd, dims, &dev);
+        if (hhc::handle_radius(h) != 1) return STENCIL_EINVAL;   // slabs: radius-1 kinds (ring of one row)
         rank = rk; world = wd; g = gg;
         if (int rc = partition(dims[0], rank, world, g, &part)) return rc;
         inner = dims[1] * dims[2];

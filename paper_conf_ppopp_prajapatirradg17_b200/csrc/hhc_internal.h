@@ -32,15 +32,26 @@ struct HexParams {
     float c;                // Eq. 1 constant
     float kappa;            // Gradient-2D
     int compute_only;       // K4: skip all global<->shared transfers (Citer micro-benchmark)
+    int R;                  // stencil radius = fixed-ring width (1; 2-4 for the f4 kinds, 1D)
 };
+
+// Radius of a kind's neighbourhood (1D binomial smoothers of radius 2-4).
+inline int kind_radius(int kind) {
+    return kind == STENCIL_BINOM1D_R2 ? 2 : kind == STENCIL_BINOM1D_R3 ? 3 : kind == STENCIL_BINOM1D_R4 ? 4 : 1;
+}
 
 // Shared-memory bytes of the HHC kernels (DESIGN.md §Kernels K1/K2): two parity
 // planes in skewed coordinates, a double-buffered skewed face and the
 // per-level footprint geometry table.
-inline int64_t smem_bytes(int ndims, int tT, int tS1, int tS2, int tS3) {
+inline int64_t smem_bytes(int ndims, int tT, int tS1, int tS2, int tS3, int R = 1) {
     const int64_t NX = tS1 + tT + 2;
     const int64_t geo = 16 * (int64_t)tT;              // per-level geometry table (ints)
-    if (ndims == 1) return 4 * (2 * ((NX + 3) & ~3) + geo);   // K0: two 16-B padded planes of NX values + geometry
+    if (ndims == 1) {
+        // K0: two planes of NX1 = tS1 + R tT + 2R values, each with 4 guard floats in
+        // front and >= 8 behind (aligned 4-chunk windows), + the geometry table
+        const int64_t NX1 = tS1 + (int64_t)R * tT + 2 * R;
+        return 4 * (2 * (((NX1 + 8 + 3) & ~3) + 4) + geo);
+    }
     if (ndims == 2) return 4 * ((2 * NX + 1) * (tS2 + 8) + 2 * (int64_t)tT * NX * 2 + geo + NX + 2 * (int64_t)tT + 2 + 2 * NX);
     return 4 * (2 * NX * (tS2 + 2) * (tS3 + 4) + 2 * (int64_t)tT * NX * (tS2 + 2) * 2 + geo);
 }
@@ -60,11 +71,12 @@ inline int column_threads(int ndims, int tS2, int tS3) {
 typedef void (*hex_kernel_t)(HexParams);
 hex_kernel_t get_hex_kernel(int ndims, int kind, int mode, bool has_c, bool defw, int s2);
 int hex_kernel_regs(int ndims, int kind, int mode, bool has_c, bool defw, int s2);
-void launch_copy_ring(const float* in, float* out, int64_t S1, int64_t S2, int64_t S3, void* stream);
+void launch_copy_ring(const float* in, float* out, int64_t S1, int64_t S2, int64_t S3, void* stream, int R = 1);
 void launch_copy_full(const float* in, float* out, int64_t n, void* stream);
 
 void set_compute_only(stencil_t h, int on);
 void set_last_launches(stencil_t h, int64_t n);
+int handle_radius(stencil_t h);
 void handle_info(stencil_t h, int* kind, int* ndims, int64_t* dims, int* device);
 int handle_clone(stencil_t h, const int64_t* dims, int maxJ, stencil_t* out);
 

@@ -17,12 +17,16 @@ namespace {
 
 inline int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
 
+// Stencil radius of the kind being modelled (1; 2-4 for the f4 kinds, reading F4:
+// slopes, pitch, footprints and facets scale by R), set by model_predict.
+thread_local int64_t g_R = 1;
+
 int ndims_of(int kind) {
     switch (kind) {
     case STENCIL_JACOBI2D_5PT: case STENCIL_HEAT2D_9PT: case STENCIL_GRADIENT2D:
     case STENCIL_LAPLACIAN2D_5PT: return 2;
     case STENCIL_HEAT3D_7PT: case STENCIL_LAPLACIAN3D_27PT: return 3;
-    case STENCIL_JACOBI1D_3PT: return 1;
+    case STENCIL_JACOBI1D_3PT: case STENCIL_BINOM1D_R2: case STENCIL_BINOM1D_R3: case STENCIL_BINOM1D_R4: return 1;
     default: return 0;
     }
 }
@@ -41,13 +45,14 @@ double talg_paper_1d(const int64_t* S, int64_t T, const stencil_tile& tl, const 
     const int64_t tT = tl.t, tS = tl.s1, S1 = S[0];
     const int64_t r = T - (T / tT) * tT;
     const int64_t Nw = 2 * cdiv(T, tT) + ((r > 0 && 2 * r <= tT) ? 0 : 1);      // Eq. 3
-    const int64_t wtile = tS + tT - 2;                                          // Eq. 4
-    const int64_t w = cdiv(S1, 2 * tS + tT);                                    // Eq. 5
-    const double m_prime = 2.0 * (double)(tS + 2 * tT) * hw.L_s_per_word + 2.0 * hw.tau_sync_s;   // Eqs. 7-8
+    const int64_t R = g_R;                                                      // reading F4 (f4 kinds)
+    const int64_t wtile = tS + R * (tT - 2);                                    // Eq. 4
+    const int64_t w = cdiv(S1, 2 * tS + R * tT);                                // Eq. 5
+    const double m_prime = 2.0 * (double)(tS + 2 * R * tT) * hw.L_s_per_word + 2.0 * hw.tau_sync_s;   // Eqs. 7-8
     double sum = 0.0;
-    for (int64_t x = tS; x <= wtile; x += 2) sum += (double)cdiv(x, hw.n_v);
+    for (int64_t x = tS; x <= wtile; x += 2 * R) sum += (double)cdiv(x, hw.n_v);
     const double c = 2.0 * hw.C_iter_s * sum + (double)tT * hw.tau_sync_s;       // Eq. 9
-    const int64_t Mbytes = 4 * 2 * (tS + tT);                                    // Mtile = 2(wtile + 2)
+    const int64_t Mbytes = 4 * 2 * (wtile + 2 * R);                              // Mtile = 2(wtile + 2R)
     if (Mbytes > hw.m_block_bytes) return std::numeric_limits<double>::infinity();
     const int64_t k = std::min<int64_t>(hw.m_sm_bytes / Mbytes, hw.mtb_sm);     // Eq. 11 (reading M4)
     if (k < 1) return std::numeric_limits<double>::infinity();
@@ -92,7 +97,7 @@ double talg_paper(int nd, const int64_t* S, int64_t T, const stencil_tile& tl, c
 }
 
 // ---------------------------------------------------------------- EXACT
-inline int64_t row_width(int64_t tau, int64_t tS1, int64_t tT) { return tS1 + 2 * std::min(tau, tT - tau); }
+inline int64_t row_width(int64_t tau, int64_t tS1, int64_t tT) { return tS1 + 2 * g_R * std::min(tau, tT - tau); }
 
 int default_threads(int nd, const stencil_tile& t) {
     const int base = hhc::column_threads(nd, t.s2, t.s3);
@@ -117,14 +122,15 @@ int64_t k_exact(int64_t Mtile, int64_t threads, const model_hw_params& hw) {
 double talg_exact(int nd, const int64_t* S, int64_t T, const stencil_tile& tl, const model_hw_params& hw) {
     const int64_t tT = tl.t, tS1 = tl.s1, tS2 = tl.s2, tS3 = nd == 3 ? tl.s3 : 1;
     const int64_t S1 = S[0], S2 = S[1], S3 = nd == 3 ? S[2] : 1;
-    const int64_t Mtile = hhc::smem_bytes(nd, (int)tT, (int)tS1, (int)tS2, (int)tS3);
+    const int64_t R = g_R;
+    const int64_t Mtile = hhc::smem_bytes(nd, (int)tT, (int)tS1, (int)tS2, (int)tS3, (int)R);
     const int threads = hw.threads > 0 ? hw.threads : default_threads(nd, tl);
     if (Mtile > hw.m_block_bytes || threads > hhc::max_block_threads(nd)) return std::numeric_limits<double>::infinity();
     const int64_t k = k_exact(Mtile, threads, hw);                                       // Eq. 11
     if (k < 1) return std::numeric_limits<double>::infinity();
     const int64_t G = nd == 1 ? 1 : std::max<int64_t>(1, threads / hhc::column_threads(nd, (int)tS2, (int)tS3));
-    const int64_t P = 2 * tS1 + tT, h = tT / 2;
-    const int64_t wA = cdiv(S1 + h, P);                        // reading G2
+    const int64_t P = 2 * tS1 + R * tT, h = tT / 2;
+    const int64_t wA = cdiv(S1 + R * h, P);                    // reading G2 (F4: radius R)
     const int64_t wB = S1 > tS1 ? cdiv(S1 - tS1, P) : 0;
     const double L_sm = hw.L_s_per_word * hw.n_sm;             // reading M5
     const int64_t Nw = cdiv(2 * T, tT) + 1;
@@ -151,10 +157,10 @@ double talg_exact(int nd, const int64_t* S, int64_t T, const stencil_tile& tl, c
         for (int64_t tau = lo; tau < hi; ++tau) {
             const int64_t W = row_width(tau, tS1, tT);
             area += W;
-            if (tau == lo) reads += W + 2;
-            else if (tau <= h) reads += 4;
+            if (tau == lo) reads += W + 2 * R;
+            else if (tau <= h) reads += 4 * R;
             if (t0 + tau == T || tau == hi - 1) writes += W;
-            else if (tau + 1 > h) writes += 4;
+            else if (tau + 1 > h) writes += 4 * R;
             // reading M9 (geometry 2): the G x-groups split the row, so a level lasts
             // G*ceil(W/G) rows' worth of the block's vector units
             const int64_t We = (hw.geometry == 2 && G > 1) ? G * cdiv(W, G) : W;
@@ -245,10 +251,14 @@ extern "C" double model_predict(stencil_kind kind, int ndims, const int64_t* dim
         if (dims[d] < 3) return nan;
     if (!tile_ok(ndims, tile)) return nan;
     if (hw->n_sm < 1 || hw->n_v < 1 || hw->mtb_sm < 1 || hw->m_sm_bytes < 1 || hw->m_block_bytes < 1) return nan;
-    int64_t S[3] = {dims[0] - 2, ndims >= 2 ? dims[1] - 2 : 1, ndims == 3 ? dims[2] - 2 : 1};
+    const int R = hhc::kind_radius(kind);
+    if (dims[0] < 2 * R + 1) return nan;
+    int64_t S[3] = {dims[0] - 2 * R, ndims >= 2 ? dims[1] - 2 : 1, ndims == 3 ? dims[2] - 2 : 1};
     auto f = hw->geometry >= 1 ? talg_exact : talg_paper;
-    if (hw->n_gpus > 1) return talg_dist(ndims, S, T, tile, *hw, f);
-    return f(ndims, S, T, tile, *hw);
+    g_R = R;
+    const double v = (hw->n_gpus > 1 && R == 1) ? talg_dist(ndims, S, T, tile, *hw, f) : f(ndims, S, T, tile, *hw);
+    g_R = 1;
+    return v;
 }
 
 // Wavefront-parallel Jacobi-1D: "the total execution time is
@@ -341,7 +351,9 @@ extern "C" int model_select_tile(stencil_kind kind, int ndims, const int64_t* di
     for (int d = 0; d < ndims; ++d)
         if (dims[d] < 3) return STENCIL_EINVAL;
     // search space, reading M6
-    const int64_t S1 = dims[0] - 2, S2 = ndims >= 2 ? dims[1] - 2 : 1, S3 = ndims == 3 ? dims[2] - 2 : 1;
+    const int64_t S1 = dims[0] - 2 * hhc::kind_radius(kind), S2 = ndims >= 2 ? dims[1] - 2 : 1,
+                  S3 = ndims == 3 ? dims[2] - 2 : 1;
+    if (S1 < 1) return STENCIL_EINVAL;
     const int64_t Tev = T + (T & 1);
     const int64_t tTmax = std::min<int64_t>(Tev, 128), tS1max = std::min<int64_t>(S1, 64);
     const int64_t innerS = ndims == 2 ? S2 : S3;

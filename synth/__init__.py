@@ -22,7 +22,7 @@ _M64 = np.uint64(0xFFFFFFFFFFFFFFFF)
 _SEED_MIX = 0xD1B54A32D192ED03
 
 # Per-config seeds: C1..C5 -> 1..5
-CONFIG_SEEDS = {"C1": 1, "C2": 2, "C3": 3, "C4": 4, "C5": 5, "X1": 7, "W1": 8}
+CONFIG_SEEDS = {"C1": 1, "C2": 2, "C3": 3, "C4": 4, "C5": 5, "X1": 7, "W1": 8, "X2": 9}
 
 
 def _splitmix64(x: np.ndarray) -> np.ndarray:

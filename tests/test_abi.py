@@ -271,3 +271,30 @@ def test_leff_fit_recovers_L(lib):
             full.append((dims, T, tile, t))
     fit = tune.fit_leff(cal, 4, full)
     assert abs(fit["L_s_per_word"] / Lstar - 1) < 1e-3 and fit["rel_rmse"] < 1e-3 and fit["n"] == len(full)
+
+
+@pytest.mark.parametrize("geometry", [hhc.PAPER, hhc.EXACT])
+def test_model_radius_r_matches_oracle(lib, geometry):
+    """f4 kinds (radius R = 2..4, reading F4): C++ model_predict vs the oracle,
+    random problems and tiles; model_select_tile's argmin and candidates too."""
+    rnd = random.Random(90 + geometry)
+    n = 0
+    for _ in range(150):
+        kind = rnd.choice([8, 9, 10])
+        R = hhc.KIND_RADIUS[kind]
+        o, c = hw_pair(kind if kind < 7 else 1, geometry, rnd, b200=True)
+        S = rnd.randint(50, 200000)
+        tile = (2 * rnd.randint(1, 64), rnd.randint(1, 3000), 0, 0)
+        T = rnd.randint(1, 500)
+        got = hhc.model_predict(kind, (S + 2 * R,), T, tile, c)
+        exp = mo.talg(1, (S,), T, tile, o, R)
+        if math.isinf(exp):
+            assert math.isinf(got)
+        else:
+            n += 1
+            assert abs(got - exp) <= 1e-12 * exp, (kind, S, T, tile, got, exp)
+    assert n > 50
+    o, c = hw_pair(1, geometry, b200=True)
+    best, thr, cands = hhc.model_select_tile(9, (5000 + 6,), 64, c, 0.10)
+    ob, ot, oc = mo.select_tile(1, (5000,), 64, o, 0.10, R=3)
+    assert best == ob and cands == oc

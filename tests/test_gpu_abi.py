@@ -24,7 +24,8 @@ CASES = [(hhc.HEAT2D_9PT, (32, 12, 512, 0), 384), (hhc.HEAT2D_9PT, (16, 20, 128,
          (hhc.GRADIENT2D, (8, 3, 256, 0), 128), (hhc.JACOBI2D_5PT, (4, 2, 32, 0), 16),
          (hhc.HEAT3D_7PT, (8, 8, 16, 64), 512), (hhc.HEAT3D_7PT, (4, 2, 2, 32), 64),
          (hhc.LAPLACIAN3D_27PT, (8, 6, 8, 64), 256), (hhc.LAPLACIAN3D_27PT, (2, 1, 1, 32), 8),
-         (hhc.JACOBI1D_3PT, (128, 2048, 0, 0), 256), (hhc.JACOBI1D_3PT, (8, 64, 0, 0), 256)]
+         (hhc.JACOBI1D_3PT, (128, 2048, 0, 0), 256), (hhc.JACOBI1D_3PT, (8, 64, 0, 0), 256),
+         (hhc.BINOM1D_R3, (64, 4096, 0, 0), 256)]
 
 
 @pytest.mark.parametrize("kind,tile,threads", CASES)
@@ -32,7 +33,7 @@ def test_exact_k_equals_hardware_occupancy(kind, tile, threads):
     nd = hhc.KIND_NDIMS[kind]
     smem, thr, regs = hhc.stencil_tile_resources(nd, tile, threads, kind=kind)
     assert regs > 0 and thr == threads
-    assert smem == mo.smem_bytes_exact(nd, tile)
+    assert smem == mo.smem_bytes_exact(nd, tile, hhc.KIND_RADIUS.get(kind, 1))
     props = torch.cuda.get_device_properties(0)
     hw = mo.HW(nSM=props.multi_processor_count, nV=128, MTBSM=32, RSM=65536, MSM=228 * 1024,
                Mblock=227 * 1024, L=1e-12, tau_sync=1e-9, T_sync=1e-6, C_iter=1e-9, regs_per_thread=regs,

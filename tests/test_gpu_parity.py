@@ -222,6 +222,31 @@ def test_parity_1d(mode):
             assert_bits(got, exp, f"1D n {n} T {T} tile {tile}")
 
 
+@pytest.mark.parametrize("kind", [hhc.BINOM1D_R2, hhc.BINOM1D_R3, hhc.BINOM1D_R4])
+@pytest.mark.parametrize("mode", [hhc.PLAIN, hhc.FUSED])
+def test_parity_radius_r_1d(kind, mode):
+    """radius-R hexagons (slope R, pitch 2 tS1 + R tT, ring of
+    width R, 2R-row footprints/facets) in K0, bit-exact against the oracle on
+    random sizes, tiles (grids smaller than a tile included) and T."""
+    rng = np.random.default_rng(200 + 10 * kind + mode)
+    R = hhc.KIND_RADIUS[kind]
+    for tile in [(2, 1), (4, 3), (8, 32), (16, 100), (64, 512), (6, 2000), (32, 4096)]:
+        n = int(rng.integers(2 * R + 1, 7000))
+        a = field(int(rng.integers(1, 1 << 30)), (n,))
+        for T in (1, 2, 7, tile[0] + 1, 3 * tile[0] + 5):
+            exp = oracle.run(kind, a, T, mode)
+            got = gpu_run(kind, a, T, tile, mode)
+            assert_bits(got, exp, f"radius {R} n {n} T {T} tile {tile}")
+    a = field(301, (50001,))
+    offs, w = oracle.stencil_info(kind)
+    coeffs = [float(x) * 0.97 for x in w] + [0.002]
+    assert_bits(gpu_run(kind, a, 37, (8, 512), mode, coeffs=coeffs),
+                oracle.run(kind, a, 37, mode, coeffs=coeffs), "radius coeffs")
+    if mode == hhc.FUSED:
+        plain = oracle.run(kind, a, 100, hhc.PLAIN)
+        assert max_rel(gpu_run(kind, a, 100, (32, 2048), hhc.FUSED), plain) <= 1e-5
+
+
 def test_parity_1d_large_and_coeffs():
     a = field(71, (1_000_003,))
     for T, tile in ((100, (32, 2048)), (257, (64, 4096))):

@@ -280,3 +280,50 @@ def test_xgroup_rows_reading_m9():
             assert tg >= te
             larger += tg > te
     assert larger >= 1
+
+
+# ---- radius R (reading F4)
+def test_radius_r_tiling_geometry():
+    """Brute force with radius R: exact cover, every dependence (t-1, x-R..x+R)
+    from the same tile or an earlier row, per-row hexagon counts and the
+    interior footprints tS1 + 2R tT + 2R (reads) / tS1 + 2R tT - 2R (facets)."""
+    for R in (2, 3):
+        for tT in (2, 4, 6):
+            for tS in (1, 3, 5):
+                S1, T = 90, 3 * tT + 1
+                rows, w, reads, writes, tiles = hg.analyse(S1, T, tS, tT, R)
+                wA, wB = mo.w_rows_exact(S1, tS, tT, R)
+                for m in rows[1:-1]:
+                    assert w[m] == (wA if m % 2 == 0 else wB), (R, tT, tS, m)
+                for (m, j), pts in tiles.items():
+                    ts = {t for t, _ in pts}
+                    xs = {x for _, x in pts}
+                    if len(pts) != sum(mo.row_width(t, tS, tT, R) for t in range(tT)):
+                        continue
+                    if min(xs) < 2 * R + 1 or max(xs) > S1 - 2 * R or min(ts) < 2 or max(ts) >= T:
+                        continue
+                    r, wr = mo.row_io_exact(tS, tT, 0, tT, min(ts), T, R)
+                    assert reads[(m, j)] == r == tS + 2 * R * tT + 2 * R, (R, tT, tS)
+                    assert writes[(m, j)] == wr == tS + 2 * R * tT - 2 * R, (R, tT, tS)
+
+
+def test_radius_r_paper_model_hand_example():
+    """Section 4.1's 1D model with reading F4 at R = 2 on the GTX 980 constants
+    (Citer of Jacobi2D as a stand-in), S = 4096, T = 64, tile (tT, tS) = (8, 64):
+      Nw = 2*8 + 1 = 17                           (Eq. 3, T mod tT = 0)
+      wtile = 64 + 2*(8-2) = 76                   (Eq. 4, slope 2)
+      w = ceil(4096 / (128 + 16)) = 29            (Eq. 5, pitch 2 tS + R tT)
+      m' = 2*(64 + 32)*2.944e-11 + 2*7.96e-10 = 7.24448e-9 s      (Eqs. 7-8)
+      c = 2*3.39e-8*(1+1+1+1) + 8*7.96e-10 = 2.77568e-7 s         (Eq. 9, x = 64, 68, 72, 76)
+      Mtile = 2*(76 + 4) = 160 words = 640 B -> k = min(98304/640, 32) = 32   (Eq. 11)
+      Ttile = m' + c + 31*max(m', c) = 7.24448e-9 + 32*2.77568e-7 = 8.88942048e-6 s  (Eq. 12)
+      rounds = ceil(ceil(29/32)/16) = 1
+      Talg = 17*8.88942048e-6 + 17*9.24e-7 = 1.6682814816e-4 s    (Eq. 6)"""
+    hw = mo.gtx980(1)
+    t = mo.talg(1, (4096,), 64, (8, 64, 0, 0), hw, R=2)
+    mp = 2 * (64 + 32) * hw.L + 2 * hw.tau_sync
+    c = 2 * hw.C_iter * 4 + 8 * hw.tau_sync
+    assert math.isclose(mp, 7.24448e-9, rel_tol=1e-12) and math.isclose(c, 2.77568e-7, rel_tol=1e-12)
+    assert math.isclose(t, 1.6682814816e-4, rel_tol=1e-11), t
+    # R = 1 is the printed model
+    assert mo.talg(1, (4096,), 64, (8, 64, 0, 0), hw, R=1) == mo.talg(1, (4096,), 64, (8, 64, 0, 0), hw)

@@ -6,6 +6,7 @@ defines the iteration; R1-R4 fix the stencil bodies, the ring and
 the expression order.  No GPU needed."""
 from fractions import Fraction
 
+import math
 import numpy as np
 import pytest
 
@@ -365,3 +366,62 @@ def test_jacobi1d_fused_vs_plain_and_threads():
     f = oracle.run(oracle.JACOBI1D_3PT, a, 64, FUSED)
     assert np.max(np.abs(f.astype(np.float64) - p) / np.maximum(np.abs(p), 2.0 ** -10)) <= 1e-5
     assert np.array_equal(oracle.run(oracle.JACOBI1D_3PT, a, 64, FUSED, nthreads=1), f)
+
+
+# ---- radius-r 1D binomial smoothers (kinds 8-10)
+@pytest.mark.parametrize("kind,R", [(8, 2), (9, 3), (10, 4)])
+def test_radius_r_hand_values_and_ring(kind, R):
+    """T = 1 by hand: binomial weights C(2R, k)/4^R on x^2 give
+    E[(x+D)^2] = x^2 + Var(D) = x^2 + R/2 exactly (D = centred Binomial(2R, 1/2));
+    the ring (R cells each side) is untouched."""
+    a = (np.arange(3 * R + 8, dtype=np.float32)) ** 2
+    out = oracle.run(kind, a, 1, oracle.FUSED)
+    x = np.arange(a.size, dtype=np.float64)
+    inner = slice(R, a.size - R)
+    assert np.array_equal(out[inner], (x ** 2 + R / 2.0)[inner].astype(np.float32))
+    assert np.array_equal(out[:R], a[:R]) and np.array_equal(out[-R:], a[-R:])
+    offs, w = oracle.stencil_info(kind)
+    assert offs[:, 0].tolist() == list(range(-R, R + 1))
+    assert np.array_equal(w.astype(np.float64) * 4 ** R, [math.comb(2 * R, k) for k in range(2 * R + 1)])
+
+
+@pytest.mark.parametrize("kind,R", [(8, 2), (9, 3), (10, 4)])
+def test_radius_r_fourier_mode(kind, R):
+    """Binomial smoothing has the closed-form symbol lambda = cos(theta/2)^(2R):
+    a sine mode vanishing on the ring decays by lambda^T (the ring of width R
+    holds the mode's exact values, which equal the periodic continuation only
+    at the zero-crossings, so the comparison stays outside the ring's cone of
+    influence, R*T cells from each end)."""
+    S, T = 4001, 40
+    p = 400
+    th = math.pi * p / (S - 1)
+    x = np.arange(S)
+    u0 = np.sin(th * x).astype(np.float32)
+    lam = math.cos(th / 2) ** (2 * R)
+    got = oracle.run(kind, u0, T, oracle.FUSED).astype(np.float64)
+    # points farther than R*T from both ends only see the sine (odd extension of
+    # sin(theta x) about x = 0 and x = S-1 continues it exactly)
+    core = slice(R * T + R, S - R * T - R)
+    assert np.max(np.abs(got[core] - lam ** T * np.sin(th * x[core]))) <= (4 * T * (2 * R + 1) + 2) * 2.0 ** -24
+    assert lam ** T < 0.5                          # the identity map would fail the check above
+
+
+@pytest.mark.parametrize("kind,R", [(8, 2), (10, 4)])
+def test_radius_r_dense_matrix_and_affine(kind, R):
+    """Independent check of the loop: a dense fp64 iteration matrix (ring rows
+    identity), x_T = M^T x_0 within 4 T |N| 2^-24 max|x|; and an affine field
+    with short mantissas is an exact fixed point (symmetric dyadic weights)."""
+    from synth import field
+    S, T = 23, 7
+    a = field(5, (S,))
+    offs, w = oracle.stencil_info(kind)
+    M = np.eye(S)
+    for i in range(R, S - R):
+        M[i, :] = 0.0
+        for o, wj in zip(offs[:, 0], w.astype(np.float64)):
+            M[i, i + o] += wj
+    ref = np.linalg.matrix_power(M, T) @ a.astype(np.float64)
+    got = oracle.run(kind, a, T, oracle.FUSED).astype(np.float64)
+    assert np.max(np.abs(got - ref)) <= 4 * T * len(w) * 2.0 ** -24 * np.max(np.abs(a))
+    aff = (3.0 + 2.0 * np.arange(S)).astype(np.float32)
+    assert np.array_equal(oracle.run(kind, aff, T, oracle.PLAIN), aff)
