@@ -370,6 +370,14 @@ def sweep(args):
                                                              tile=tile))
         pts.append(p)
         print(json.dumps(p), flush=True)
+        if len(pts) % 200 == 0:            # partial results survive a killed job
+            summarise_sweep(args, kind, dims, T, cal, pts, None, None, None, final=False)
+    summarise_sweep(args, kind, dims, T, cal, pts, h, d_in, d_out, final=True)
+
+
+def summarise_sweep(args, kind, dims, T, cal, pts, h, d_in, d_out, final=True):
+    """RMSE per predictor over all points and the near-best subset (reading Q15);
+    with final=True also the chosen-tile gaps of the model argmins (reading Q17)."""
     best = min(pts, key=lambda p: p["texec"])
     res = {"config": args.config, "n_points": len(pts), "best_measured": best, "points": pts}
     for name in ("talg_paper", "talg_exact", "talg_exactg", "talg_exact_leff"):
@@ -378,8 +386,8 @@ def sweep(args):
         ra, rn, nn = stats(pts, name)
         res[name] = {"rmse_all": ra, "rmse_within_20pct": rn, "n_within_20pct": nn}
     # chosen-tile gaps (reading Q17), model argmin over the swept points and over Eq. 31's space
-    for geom, name, lf in ((hhc.PAPER, "paper", False), (hhc.EXACT, "exact", False), (hhc.EXACT_G, "exactg", False),
-                           (hhc.EXACT, "exact_leff", True)):
+    for geom, name, lf in (() if not final else ((hhc.PAPER, "paper", False), (hhc.EXACT, "exact", False), (hhc.EXACT_G, "exactg", False),
+                           (hhc.EXACT, "exact_leff", True))):
         if lf and not (cal.get("exact_leff") or {}).get(str(kind)):
             continue
         hw = b200_hw(cal, kind, geom, leff=lf)
@@ -394,7 +402,32 @@ def sweep(args):
     out = args.out or os.path.join(ROOT, "profiles", "r02", f"sweep_{args.config}.json")
     with open(out, "w") as f:
         json.dump(res, f, indent=1)
-    print(json.dumps({k: v for k, v in res.items() if k != "points"}))
+    if final:
+        print(json.dumps({k: v for k, v in res.items() if k != "points"}))
+
+
+def finish(args):
+    """Summarise a sweep from its points (the JSON, or the JSON lines of a sweep
+    log whose job was cut off) and measure the model argmins (reading Q17)."""
+    import torch
+
+    import bench
+    from synth import CONFIG_SEEDS, field
+    cfg = bench.CONFIGS[args.config]
+    kind, dims, T = cfg["kind"], cfg["dims"], cfg["T"]
+    cal = load_cal(args.cal)
+    src = args.src or os.path.join(ROOT, "profiles", "r02", f"sweep_{args.config}.json")
+    if src.endswith(".json"):
+        pts = json.load(open(src))["points"]
+    else:
+        pts = [json.loads(l) for l in open(src) if l.startswith('{"tile"')]
+    h = d_in = d_out = None
+    if args.measure:
+        a = field(CONFIG_SEEDS[args.config], dims)
+        d_in = torch.from_numpy(a).cuda()
+        d_out = torch.empty_like(d_in)
+        h = hhc.stencil_create(kind, dims)
+    summarise_sweep(args, kind, dims, T, cal, pts, h, d_in, d_out, final=args.measure)
 
 
 def select(args):
@@ -460,8 +493,15 @@ def main(argv=None):
     e.add_argument("--max-measure", type=int, default=100000)
     e.add_argument("--budget", type=float, default=1800.0)
     e.add_argument("--geometry", default="exact", choices=["paper", "exact", "exactg"])
+    f = sub.add_parser("finish")
+    f.add_argument("--config", default="C2")
+    f.add_argument("--cal", default=None)
+    f.add_argument("--src", default=None, help="sweep JSON or sweep log (JSON lines)")
+    f.add_argument("--out", default=None)
+    f.add_argument("--reps", type=int, default=5)
+    f.add_argument("--measure", action="store_true", help="time the model argmins on the GPU")
     args = ap.parse_args(argv)
-    {"calibrate": calibrate, "sweep": sweep, "select": select}[args.cmd](args)
+    {"calibrate": calibrate, "sweep": sweep, "select": select, "finish": finish}[args.cmd](args)
 
 
 if __name__ == "__main__":
