@@ -267,6 +267,30 @@ def fit_exact(kind, insts, geometry=None):
     return {"C_iter_s": c, "tau_level_s": tau, "rel_rmse": err, "n": len(rows)}
 
 
+def near_space(nd, kind, dims, T):
+    """The region of SURVEY §8(d)'s space where the full sweep found its best
+    tiles (2D: tT 16..48, tS1 6..24, tS2 256..768; 3D: tT 4..12, tS1 2..12,
+    tS2 4..16, tS3 32..128), shuffled (seed 13): densifies the near-best subset
+    the RMSE of reading Q15 is taken over."""
+    out = []
+    if nd == 2:
+        tiles = [(tT, tS1, tS2, 0) for tT in range(16, min(48, T + T % 2) + 1, 2) for tS1 in range(6, 25)
+                 for tS2 in range(256, 769, 32)]
+    else:
+        tiles = [(tT, tS1, tS2, tS3) for tT in range(4, 13, 2) for tS1 in range(2, 13) for tS2 in range(4, 17)
+                 for tS3 in (32, 64, 96, 128)]
+    for t in tiles:
+        base = t[2] // 8 if nd == 2 else (t[3] // 4) * t[2]
+        for g in (2, 3, 4, 6):
+            try:
+                hhc.stencil_tile_resources(nd, t, base * g, kind=kind)
+            except hhc.StencilError:
+                continue
+            out.append((t, base * g))
+    random.Random(13).shuffle(out)
+    return out
+
+
 def full_space(nd, kind, dims, T):
     """SURVEY §8(d)'s sweep space pruned by the shared-memory limit: 2D tT in
     2..64 even, tS1 in 1..64, tS2 in 32..1024 step 32, threads = column
@@ -347,7 +371,8 @@ def sweep(args):
     h = hhc.stencil_create(kind, dims)
     pts = []
     t_start = time.time()
-    space = full_space(nd, kind, dims, T) if args.space == "full" else sweep_tiles(nd, 10 ** 9)
+    space = (full_space(nd, kind, dims, T) if args.space == "full" else
+             near_space(nd, kind, dims, T) if args.space == "near" else sweep_tiles(nd, 10 ** 9))
     best_t = math.inf
     for tile, threads in space[:args.limit]:
         if time.time() - t_start > args.budget:
@@ -416,11 +441,18 @@ def finish(args):
     cfg = bench.CONFIGS[args.config]
     kind, dims, T = cfg["kind"], cfg["dims"], cfg["T"]
     cal = load_cal(args.cal)
-    src = args.src or os.path.join(ROOT, "profiles", "r02", f"sweep_{args.config}.json")
-    if src.endswith(".json"):
-        pts = json.load(open(src))["points"]
-    else:
-        pts = [json.loads(l) for l in open(src) if l.startswith('{"tile"')]
+    srcs = args.src or [os.path.join(ROOT, "profiles", "r02", f"sweep_{args.config}.json")]
+    pts, seen = [], set()
+    for src in srcs:
+        if src.endswith(".json"):
+            new = json.load(open(src))["points"]
+        else:
+            new = [json.loads(l) for l in open(src) if l.startswith('{"tile"')]
+        for p in new:
+            key = (tuple(p["tile"]), p["threads"])
+            if key not in seen:              # a tile measured twice keeps its first sweep's time
+                seen.add(key)
+                pts.append(p)
     h = d_in = d_out = None
     if args.measure:
         a = field(CONFIG_SEEDS[args.config], dims)
@@ -483,7 +515,7 @@ def main(argv=None):
     s.add_argument("--limit", type=int, default=400)
     s.add_argument("--reps", type=int, default=5)
     s.add_argument("--budget", type=float, default=900.0)
-    s.add_argument("--space", default="grid", choices=["grid", "full"])
+    s.add_argument("--space", default="grid", choices=["grid", "full", "near"])
     e = sub.add_parser("select")
     e.add_argument("--config", default="C2")
     e.add_argument("--cal", default=None)
@@ -496,7 +528,7 @@ def main(argv=None):
     f = sub.add_parser("finish")
     f.add_argument("--config", default="C2")
     f.add_argument("--cal", default=None)
-    f.add_argument("--src", default=None, help="sweep JSON or sweep log (JSON lines)")
+    f.add_argument("--src", default=None, nargs="+", help="sweep JSONs or sweep logs (JSON lines), merged")
     f.add_argument("--out", default=None)
     f.add_argument("--reps", type=int, default=5)
     f.add_argument("--measure", action="store_true", help="time the model argmins on the GPU")
