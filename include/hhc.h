@@ -240,6 +240,28 @@ int stencil_run_dist(stencil_t h, void* comm, const float* d_in_slab, float* d_o
 int stencil_run_dist_local(stencil_t h, int world, const float* d_in, float* d_out, int64_t T,
                            stencil_tile tile, int threads, int overlap, void* cuda_stream);
 
+/* ---- non-redundant, hexagon-aligned multi-GPU decomposition (2D
+ * kinds).  Hexagons go to ranks by their centre column (owned rows [b0, b1) =
+ * the slab partition); every point is computed once.  A rank stores the global
+ * rows [x_lo, x_hi) = [b0 - H, b1 + H) (H = tS1/2 + tT/2 + 3) its hexagons touch;
+ * the K1 kernel writes each facet row (reading G3: a value some other hexagon
+ * reads) that a neighbour also stores straight into the neighbour's plane (peer
+ * stores from the edge CTAs, fused with the compute).  Rows of hexagons run in
+ * order on all ranks (a row reads only earlier rows). */
+
+/* part[0..5] = b0, b1, x_lo, x_hi, held_lo, held_hi of `rank` (host only);
+ * STENCIL_ETILE if a slab holds fewer than 2H rows (a hexagon would reach two
+ * ranks away). */
+int stencil_hexdist_partition(int64_t S1, int rank, int world, stencil_tile tile, int64_t part[6]);
+
+/* The f1 decomposition with `world` virtual ranks of ONE device (separate
+ * planes per rank, peer stores = device stores into the neighbour's planes):
+ * A_T from A_0 like stencil_run (full-grid device in/out, no overlap), 2D
+ * handles only.  Synchronises.  stencil_last_launches(h) = the kernel launches
+ * (rows x ranks). */
+int stencil_run_hexdist_local(stencil_t h, int world, const float* d_in, float* d_out, int64_t T,
+                              stencil_tile tile, int threads, void* cuda_stream);
+
 /* Measurement helper (bench.py roofline): run like stencil_run but without the
  * CUDA graph, with a CUDA event pair around every hexagon-row launch on
  * cuda_stream; synchronises and returns the summed device time of the HHC

@@ -137,6 +137,9 @@ def load(build_if_missing: bool = False):
     lib.stencil_run_dist.argtypes = [vp, vp, vp, vp, ctypes.c_int64, stencil_tile, ctypes.c_int, vp]
     lib.stencil_run_dist_local.argtypes = [vp, ctypes.c_int, vp, vp, ctypes.c_int64, stencil_tile, ctypes.c_int,
                                            ctypes.c_int, vp]
+    lib.stencil_hexdist_partition.argtypes = [ctypes.c_int64, ctypes.c_int, ctypes.c_int, stencil_tile, i64p]
+    lib.stencil_run_hexdist_local.argtypes = [vp, ctypes.c_int, vp, vp, ctypes.c_int64, stencil_tile, ctypes.c_int,
+                                              vp]
     _lib = lib
     return lib
 
@@ -352,6 +355,19 @@ def stencil_run_dist_local(h, world: int, d_in, d_out, T: int, tile, threads: in
                                          int(threads), int(overlap), _stream(stream)), "stencil_run_dist_local")
 
 
+def stencil_hexdist_partition(S1: int, rank: int, world: int, tile):
+    """f1: (b0, b1, x_lo, x_hi, held_lo, held_hi) of one rank (host only)."""
+    out = (ctypes.c_int64 * 6)()
+    _check(load().stencil_hexdist_partition(int(S1), int(rank), int(world), make_tile(tile), out),
+           "stencil_hexdist_partition")
+    return tuple(out)
+
+
+def stencil_run_hexdist_local(h, world: int, d_in, d_out, T: int, tile, threads: int = 0, stream=None):
+    _check(load().stencil_run_hexdist_local(h.handle, int(world), _ptr(d_in), _ptr(d_out), int(T), make_tile(tile),
+                                            int(threads), _stream(stream)), "stencil_run_hexdist_local")
+
+
 def stencil_plan_info(dims, T: int, tile):
     d, nd = _dims(dims)
     out = [ctypes.c_int64() for _ in range(4)]
@@ -382,4 +398,5 @@ EXPORTED_SYMBOLS = ["stencil_create", "stencil_destroy", "stencil_run", "stencil
                     "stencil_profile", "stencil_run_wavefront", "stencil_wavefront_info",
                     "model_predict_wavefront", "model_select_wavefront_tile", "stencil_dist_get_unique_id",
                     "stencil_dist_init", "stencil_dist_set_overlap", "stencil_dist_destroy", "stencil_dist_partition",
-                    "stencil_run_dist", "stencil_run_dist_local"]
+                    "stencil_run_dist", "stencil_run_dist_local", "stencil_hexdist_partition",
+                    "stencil_run_hexdist_local"]

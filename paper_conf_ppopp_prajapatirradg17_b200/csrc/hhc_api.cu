@@ -742,3 +742,127 @@ int handle_clone(stencil_t h, const int64_t* dims, int maxJ, stencil_t* out) {
     return rc;
 }
 }
+
+// ---- f1: non-redundant, hexagon-aligned multi-GPU decomposition (2D).
+// Hexagons are assigned to ranks by their centre column (owned rows [b0, b1) of
+// the slab partition); every point is computed exactly once (no ghost rows, no
+// redundant compute).  A rank stores the global rows [b0 - H, b1 + H) its
+// hexagons touch (H = tS1/2 + tT/2 + 3: half a hexagon plus the footprint halo)
+// in planes indexed by global x.  K1 writes every facet row that a neighbour
+// also stores straight into the neighbour's plane (peer stores fused into the
+// edge CTAs, HexParams::peer), so after row m of hexagons every value row m+1
+// reads is in the reader's own planes.  Dependences: row m+1 on any rank reads
+// only values of rows <= m (reading G2), so the rows are run in order, all
+// ranks' hexagons of row m before row m+1.  stencil_run_hexdist_local runs
+// `world` virtual ranks of one device this way (peer stores = device stores
+// into the neighbour's buffers); across GPUs the same kernel stores through
+// peer-mapped (IPC) pointers over NVLink.
+namespace {
+struct HexRank {
+    int64_t b0, b1, x_lo, x_hi, held_lo, held_hi;
+    float* P[2] = {nullptr, nullptr};
+    float* Pg[2] = {nullptr, nullptr};
+};
+}  // namespace
+
+extern "C" int stencil_hexdist_partition(int64_t S1, int rank, int world, stencil_tile tile, int64_t* part) {
+    if (!part || S1 < 3 || world < 1 || rank < 0 || rank >= world || tile.t < 2 || tile.s1 < 1) return STENCIL_EINVAL;
+    const int64_t own = cdiv(S1 - 2, world);
+    const int64_t H = tile.s1 / 2 + tile.t / 2 + 3;
+    if (world > 1 && own < 2 * H) return STENCIL_ETILE;
+    const int64_t b0 = 1 + rank * own, b1 = std::min<int64_t>(1 + (rank + 1) * own, S1 - 1);
+    if (b1 <= b0) return STENCIL_EINVAL;
+    if (world > 1 && rank < world - 1 && b1 - b0 < 2 * H) return STENCIL_ETILE;
+    const int64_t v[6] = {b0, b1, std::max<int64_t>(0, b0 - H), std::min<int64_t>(S1, b1 + H),
+                          b0 - (rank == 0 ? 1 : 0), b1 + (rank == world - 1 ? 1 : 0)};
+    memcpy(part, v, sizeof(v));
+    return STENCIL_OK;
+}
+
+extern "C" int stencil_run_hexdist_local(stencil_t h, int world, const float* d_in, float* d_out, int64_t T,
+                                         stencil_tile tile, int threads, void* cuda_stream) {
+    if (!h || world < 1 || !d_in || !d_out || T < 1) return STENCIL_EINVAL;
+    if (h->sticky) return h->sticky;
+    if (h->ndims != 2) return STENCIL_EINVAL;                  // the facet peer stores are K1's
+    int G, thr;
+    if (int rc = check_tile(h->ndims, tile, threads, h->smem_optin, &G, &thr, h->kind)) return rc;
+    cudaStream_t s = (cudaStream_t)cuda_stream;
+    cudaSetDevice(h->device);
+    const int64_t S1 = h->dims[0], S2 = h->dims[1], inner = S2;
+    std::vector<HexRank> rk(world);
+    auto release = [&]() {
+        cudaStreamSynchronize(s);
+        for (auto& r : rk)
+            for (float* p : r.P)
+                if (p) cudaFree(p);
+    };
+    for (int k = 0; k < world; ++k) {
+        int64_t part[6];
+        if (int rc = stencil_hexdist_partition(S1, k, world, tile, part)) { release(); return rc; }
+        HexRank& r = rk[k];
+        r.b0 = part[0]; r.b1 = part[1]; r.x_lo = part[2]; r.x_hi = part[3]; r.held_lo = part[4]; r.held_hi = part[5];
+        const size_t bytes = (size_t)((r.x_hi - r.x_lo) * inner) * sizeof(float);
+        for (int i = 0; i < 2; ++i) {
+            if (cudaMalloc(&r.P[i], bytes) != cudaSuccess) { release(); return STENCIL_ENOMEM; }
+            r.Pg[i] = r.P[i] - r.x_lo * inner;                 // global-x indexed
+            // level 0 (and its ring) into both planes
+            cudaMemcpyAsync(r.P[i], d_in + r.x_lo * inner, bytes, cudaMemcpyDeviceToDevice, s);
+        }
+    }
+    if (int rc = prepare_rows(h, h->dims, T, tile, thr)) { release(); return rc; }
+    hex_kernel_t kern = get_hex_kernel(h->ndims, h->kind, h->mode, h->has_c, h->defw, tile.s2);
+    const int64_t smem = smem_bytes(h->ndims, tile.t, tile.s1, tile.s2, tile.s3, h->R);
+    std::vector<RowPlan> rows;
+    plan_rows(h->ndims, h->dims, T, tile, rows, h->R);
+    HexParams p;
+    memset(&p, 0, sizeof(p));
+    p.S1 = S1; p.S2 = S2; p.S3 = 1; p.T = T;
+    p.tT = tile.t; p.tS1 = tile.s1; p.tS2 = tile.s2; p.tS3 = 0;
+    p.G = G; p.P = 2 * tile.s1 + tile.t; p.R = 1; p.J = 1;
+    for (int j = 0; j < kMaxPts; ++j) p.w[j] = h->w[j];
+    p.c = h->c; p.kappa = h->kappa;
+    int64_t nl = 0;
+    for (auto& row : rows) {
+        p.t0 = row.t0; p.tau_lo = row.tau_lo; p.tau_hi = row.tau_hi; p.n2 = row.n2; p.n3 = 1;
+        for (int k = 0; k < world; ++k) {
+            const HexRank& r = rk[k];
+            // hexagons j of this row whose centre 2 x0 + tS1 lies in [2 b0, 2 b1)
+            auto first_at = [&](int64_t b) {            // smallest j with 2(xbase + jP) + tS1 >= 2b
+                const int64_t num = 2 * b - tile.s1 - 2 * row.xbase;
+                return num <= 0 ? (int64_t)0 : cdiv(num, 2 * (int64_t)p.P);
+            };
+            const int64_t jlo = k == 0 ? 0 : std::min<int64_t>(first_at(r.b0), row.w);
+            const int64_t jhi = k == world - 1 ? row.w : std::min<int64_t>(first_at(r.b1), row.w);
+            if (jhi <= jlo) continue;
+            p.xbase = row.xbase + jlo * p.P;
+            p.in = r.Pg[0];
+            p.plane[0] = r.Pg[0];
+            p.plane[1] = r.Pg[1];
+            p.npeer = world > 1;
+            for (int sd = 0; sd < 2; ++sd) {
+                const int nb = k + (sd == 0 ? -1 : 1);
+                if (nb >= 0 && nb < world) {
+                    p.peer[sd][0] = rk[nb].Pg[0]; p.peer[sd][1] = rk[nb].Pg[1];
+                    p.peer_lo[sd] = rk[nb].x_lo; p.peer_hi[sd] = rk[nb].x_hi;
+                } else {
+                    p.peer[sd][0] = p.peer[sd][1] = nullptr;
+                    p.peer_lo[sd] = p.peer_hi[sd] = 0;
+                }
+            }
+            void* args[] = {&p};
+            cudaError_t e = cudaLaunchKernel((const void*)kern, dim3((unsigned)(jhi - jlo)), dim3(thr), args,
+                                             (size_t)smem, s);
+            if (e != cudaSuccess) { release(); return cuda_fail(h, e); }
+            ++nl;
+        }
+    }
+    for (auto& r : rk) {
+        const int64_t n = (r.held_hi - r.held_lo) * inner;
+        cudaMemcpyAsync(d_out + r.held_lo * inner, r.Pg[T & 1] + r.held_lo * inner, (size_t)n * sizeof(float),
+                        cudaMemcpyDeviceToDevice, s);
+    }
+    h->last_launches = nl;
+    const int rc = cuda_fail(h, cudaGetLastError());
+    release();
+    return rc;
+}

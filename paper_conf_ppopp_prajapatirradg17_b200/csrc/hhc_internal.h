@@ -33,6 +33,12 @@ struct HexParams {
     float kappa;            // Gradient-2D
     int compute_only;       // K4: skip all global<->shared transfers (Citer micro-benchmark)
     int R;                  // stencil radius = fixed-ring width (1; 2-4 for the f4 kinds, 1D)
+    // f1, non-redundant hexagon-aligned multi-GPU (2D): the neighbour ranks' planes
+    // (indexed by global x like plane[]) and the global rows [peer_lo, peer_hi) each
+    // stores; K1 writes facet rows in those ranges into them too (peer stores)
+    int npeer;
+    float* peer[2][2];      // [side: lower x, upper x][parity]
+    int64_t peer_lo[2], peer_hi[2];
 };
 
 // Radius of a kind's neighbourhood (1D binomial smoothers of radius 2-4).

@@ -119,3 +119,23 @@ def test_product_partition_matches_reference():
                             hhc.stencil_dist_partition(S1, rank, world, g)
                         continue
                     assert hhc.stencil_dist_partition(S1, rank, world, g) == (s.r0, s.r1, s.e0, s.e1) + s.held
+
+
+def test_hexdist_partition_rules():
+    """f1 partition (host only): owned rows tile [1, S1-1) exactly, stored rows
+    extend H = tS1/2 + tT/2 + 3 on each side (clipped to the grid), the held
+    rows add the physical ring on the edge ranks, and slabs thinner than 2H are
+    rejected (a hexagon would reach two ranks away)."""
+    import paper_conf_ppopp_prajapatirradg17_b200 as hhc
+    for S1, world, tile in [(362, 4, (8, 5, 512)), (1000, 3, (16, 12, 64)), (8194, 8, (32, 12, 512))]:
+        H = tile[1] // 2 + tile[0] // 2 + 3
+        prev_b1 = 1
+        for r in range(world):
+            b0, b1, xl, xh, hl, hh = hhc.stencil_hexdist_partition(S1, r, world, tile)
+            assert b0 == prev_b1 and b1 > b0
+            assert xl == max(0, b0 - H) and xh == min(S1, b1 + H)
+            assert hl == (0 if r == 0 else b0) and hh == (S1 if r == world - 1 else b1)
+            prev_b1 = b1
+        assert prev_b1 == S1 - 1
+    with pytest.raises(hhc.StencilError):
+        hhc.stencil_hexdist_partition(100, 0, 8, (16, 12, 64))

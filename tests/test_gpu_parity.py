@@ -166,6 +166,30 @@ def test_dist_local_virtual_ranks(kind, dims, T, tT, world, overlap):
     assert_bits(d_out.cpu().numpy(), oracle.run(kind, a, T, hhc.FUSED), f"world {world} overlap {overlap}")
 
 
+@pytest.mark.parametrize("kind,dims,T,tile,world,threads", [
+    (hhc.HEAT2D_9PT, (300, 150), 37, (8, 3, 32), 2, 0),
+    (hhc.HEAT2D_9PT, (4 * 90 + 2, 700), 45, (8, 5, 512), 4, 384),
+    (hhc.GRADIENT2D, (3 * 70 + 2, 130), 21, (4, 4, 32), 3, 0),
+    (hhc.JACOBI2D_5PT, (2 * 120 + 2, 300), 64, (16, 6, 256), 2, 0),
+    (hhc.LAPLACIAN2D_5PT, (5 * 40 + 2, 90), 13, (6, 2, 64), 5, 0),
+])
+def test_hexdist_local_virtual_ranks(kind, dims, T, tile, world, threads):
+    """f1: hexagons assigned to ranks by centre column, every
+    point computed once, facets a neighbour stores written straight into its
+    planes by the edge CTAs (stencil_run_hexdist_local, virtual ranks of one
+    GPU).  The whole grid must equal the oracle bit for bit."""
+    for mode in (hhc.PLAIN, hhc.FUSED):
+        a = field(400 + kind + mode, dims)
+        s = hhc.stencil_create(kind, dims, mode=mode)
+        d_in = torch.from_numpy(a).to(DEV)
+        d_out = torch.full_like(d_in, float("nan"))
+        hhc.stencil_run_hexdist_local(s, world, d_in, d_out, T, tile, threads)
+        n = hhc.stencil_last_launches(s)
+        hhc.stencil_destroy(s)
+        assert_bits(d_out.cpu().numpy(), oracle.run(kind, a, T, mode), f"hexdist world {world} mode {mode}")
+        assert n > 0
+
+
 def test_dist_world1_nccl_free():
     """stencil_run_dist on a world-1 communicator (no NCCL needed): the slab is
     the whole grid."""
