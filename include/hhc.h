@@ -262,6 +262,26 @@ int stencil_hexdist_partition(int64_t S1, int rank, int world, stencil_tile tile
 int stencil_run_hexdist_local(stencil_t h, int world, const float* d_in, float* d_out, int64_t T,
                               stencil_tile tile, int threads, void* cuda_stream);
 
+/* f1 across processes (one per GPU, or several on one GPU for testing): this
+ * rank's planes (stored rows) and a flag pair are allocated on the current
+ * device and exported as three CUDA IPC handles (handles[192]); *out = an
+ * opaque object (free with stencil_hexdist_destroy). */
+int stencil_hexdist_create(stencil_t h, int rank, int world, stencil_tile tile, unsigned char handles[192],
+                           void** out);
+/* Open the lower (rank-1) and upper (rank+1) neighbours' handles (NULL where
+ * there is none): their planes become peer-mapped targets of K1's facet stores,
+ * their flag pair the target of this rank's row signals. */
+int stencil_hexdist_connect(stencil_t h, void* hd, const unsigned char lo[192], const unsigned char hi[192]);
+/* A_T on this rank.  d_in_stored holds level 0 of the stored rows [x_lo, x_hi),
+ * d_out_slab receives the held rows [held_lo, held_hi) (stencil_hexdist_partition).
+ * Every row of hexagons waits on the device (a spin kernel, acquire.sys) until
+ * both neighbours finished the previous row and signals its own completion
+ * (release.sys store into their flags); all ranks call it with the same T.
+ * Stream-ordered; returns before completion. */
+int stencil_run_hexdist(stencil_t h, void* hd, const float* d_in_stored, float* d_out_slab, int64_t T,
+                        int threads, void* cuda_stream);
+void stencil_hexdist_destroy(void* hd);
+
 /* Measurement helper (bench.py roofline): run like stencil_run but without the
  * CUDA graph, with a CUDA event pair around every hexagon-row launch on
  * cuda_stream; synchronises and returns the summed device time of the HHC

@@ -140,6 +140,11 @@ def load(build_if_missing: bool = False):
     lib.stencil_hexdist_partition.argtypes = [ctypes.c_int64, ctypes.c_int, ctypes.c_int, stencil_tile, i64p]
     lib.stencil_run_hexdist_local.argtypes = [vp, ctypes.c_int, vp, vp, ctypes.c_int64, stencil_tile, ctypes.c_int,
                                               vp]
+    lib.stencil_hexdist_create.argtypes = [vp, ctypes.c_int, ctypes.c_int, stencil_tile, ctypes.c_char_p, P(vp)]
+    lib.stencil_hexdist_connect.argtypes = [vp, vp, ctypes.c_char_p, ctypes.c_char_p]
+    lib.stencil_run_hexdist.argtypes = [vp, vp, vp, vp, ctypes.c_int64, ctypes.c_int, vp]
+    lib.stencil_hexdist_destroy.argtypes = [vp]
+    lib.stencil_hexdist_destroy.restype = None
     _lib = lib
     return lib
 
@@ -368,6 +373,28 @@ def stencil_run_hexdist_local(h, world: int, d_in, d_out, T: int, tile, threads:
                                             int(threads), _stream(stream)), "stencil_run_hexdist_local")
 
 
+def stencil_hexdist_create(h, rank: int, world: int, tile):
+    """f1 across processes: (opaque object, 192 bytes of IPC handles to give the neighbours)."""
+    buf = ctypes.create_string_buffer(192)
+    obj = ctypes.c_void_p()
+    _check(load().stencil_hexdist_create(h.handle, int(rank), int(world), make_tile(tile), buf, ctypes.byref(obj)),
+           "stencil_hexdist_create")
+    return obj, buf.raw
+
+
+def stencil_hexdist_connect(h, obj, lo: bytes | None, hi: bytes | None):
+    _check(load().stencil_hexdist_connect(h.handle, obj, lo, hi), "stencil_hexdist_connect")
+
+
+def stencil_run_hexdist(h, obj, d_in_stored, d_out_slab, T: int, threads: int = 0, stream=None):
+    _check(load().stencil_run_hexdist(h.handle, obj, _ptr(d_in_stored), _ptr(d_out_slab), int(T), int(threads),
+                                      _stream(stream)), "stencil_run_hexdist")
+
+
+def stencil_hexdist_destroy(obj):
+    load().stencil_hexdist_destroy(obj)
+
+
 def stencil_plan_info(dims, T: int, tile):
     d, nd = _dims(dims)
     out = [ctypes.c_int64() for _ in range(4)]
@@ -399,4 +426,5 @@ EXPORTED_SYMBOLS = ["stencil_create", "stencil_destroy", "stencil_run", "stencil
                     "model_predict_wavefront", "model_select_wavefront_tile", "stencil_dist_get_unique_id",
                     "stencil_dist_init", "stencil_dist_set_overlap", "stencil_dist_destroy", "stencil_dist_partition",
                     "stencil_run_dist", "stencil_run_dist_local", "stencil_hexdist_partition",
-                    "stencil_run_hexdist_local"]
+                    "stencil_run_hexdist_local", "stencil_hexdist_create", "stencil_hexdist_connect",
+                    "stencil_run_hexdist", "stencil_hexdist_destroy"]

@@ -866,3 +866,195 @@ extern "C" int stencil_run_hexdist_local(stencil_t h, int world, const float* d_
     release();
     return rc;
 }
+
+// ---- f1 across processes (one per GPU): the rank's planes and a flag pair are
+// exported as CUDA IPC handles, the neighbours' ones are opened (peer-mapped over
+// NVLink), K1 stores facets straight into them, and each row of hexagons waits
+// on the device until both neighbours have finished the previous row (flag
+// written by the neighbour's signal kernel with a system-scope release).
+namespace {
+__global__ void hexdist_wait_kernel(const volatile unsigned* flags, unsigned want0, unsigned want1) {
+    if (threadIdx.x == 0) {
+        while ((int)(flags[0] - want0) < 0) __nanosleep(100);
+        while ((int)(flags[1] - want1) < 0) __nanosleep(100);
+        __threadfence_system();
+    }
+}
+__global__ void hexdist_signal_kernel(unsigned* lo, unsigned* hi, unsigned v) {
+    if (threadIdx.x == 0) {
+        __threadfence_system();
+        if (lo) asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(lo), "r"(v) : "memory");
+        if (hi) asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(hi), "r"(v) : "memory");
+    }
+}
+}  // namespace
+
+struct stencil_hexdist_s {
+    int rank = 0, world = 1, device = 0;
+    stencil_tile tile{};
+    HexRank me;
+    unsigned* flags = nullptr;            // [2]: written by the lower / upper neighbour
+    float* peerP[2][2] = {{nullptr, nullptr}, {nullptr, nullptr}};   // opened IPC planes (raw)
+    unsigned* peerF[2] = {nullptr, nullptr};                         // neighbour's flag slot for me
+    int64_t peer_lo[2] = {0, 0}, peer_hi[2] = {0, 0};
+    unsigned epoch = 0;
+};
+
+extern "C" int stencil_hexdist_create(stencil_t h, int rank, int world, stencil_tile tile, unsigned char handles[192],
+                                      void** out) {
+    if (!h || !handles || !out || h->ndims != 2) return STENCIL_EINVAL;
+    *out = nullptr;
+    int64_t part[6];
+    if (int rc = stencil_hexdist_partition(h->dims[0], rank, world, tile, part)) return rc;
+    cudaSetDevice(h->device);
+    auto* d = new stencil_hexdist_s();
+    d->rank = rank; d->world = world; d->device = h->device; d->tile = tile;
+    HexRank& r = d->me;
+    r.b0 = part[0]; r.b1 = part[1]; r.x_lo = part[2]; r.x_hi = part[3]; r.held_lo = part[4]; r.held_hi = part[5];
+    const size_t bytes = (size_t)((r.x_hi - r.x_lo) * h->dims[1]) * sizeof(float);
+    cudaIpcMemHandle_t hd[3];
+    bool ok = cudaMalloc(&r.P[0], bytes) == cudaSuccess && cudaMalloc(&r.P[1], bytes) == cudaSuccess &&
+              cudaMalloc(&d->flags, 2 * sizeof(unsigned)) == cudaSuccess &&
+              cudaMemset(d->flags, 0, 2 * sizeof(unsigned)) == cudaSuccess &&
+              cudaIpcGetMemHandle(&hd[0], r.P[0]) == cudaSuccess && cudaIpcGetMemHandle(&hd[1], r.P[1]) == cudaSuccess &&
+              cudaIpcGetMemHandle(&hd[2], d->flags) == cudaSuccess;
+    if (!ok) {
+        if (r.P[0]) cudaFree(r.P[0]);
+        if (r.P[1]) cudaFree(r.P[1]);
+        if (d->flags) cudaFree(d->flags);
+        delete d;
+        cudaGetLastError();
+        return STENCIL_ECUDA;
+    }
+    for (int i = 0; i < 2; ++i) r.Pg[i] = r.P[i] - r.x_lo * h->dims[1];
+    memcpy(handles, hd, 3 * sizeof(cudaIpcMemHandle_t));
+    *out = d;
+    return STENCIL_OK;
+}
+
+// handles of the lower (rank-1) and upper (rank+1) neighbour; NULL where none
+extern "C" int stencil_hexdist_connect(stencil_t h, void* hd, const unsigned char lo[192], const unsigned char hi[192]) {
+    auto* d = static_cast<stencil_hexdist_s*>(hd);
+    if (!h || !d) return STENCIL_EINVAL;
+    cudaSetDevice(d->device);
+    const unsigned char* src[2] = {lo, hi};
+    for (int sd = 0; sd < 2; ++sd) {
+        const int nb = d->rank + (sd == 0 ? -1 : 1);
+        if (nb < 0 || nb >= d->world) continue;
+        if (!src[sd]) return STENCIL_EINVAL;
+        cudaIpcMemHandle_t hh[3];
+        memcpy(hh, src[sd], sizeof(hh));
+        void* ptr[3] = {nullptr, nullptr, nullptr};
+        for (int i = 0; i < 3; ++i)
+            if (cudaIpcOpenMemHandle(&ptr[i], hh[i], cudaIpcMemLazyEnablePeerAccess) != cudaSuccess) {
+                cudaGetLastError();
+                return STENCIL_ECUDA;
+            }
+        int64_t part[6];
+        if (int rc = stencil_hexdist_partition(h->dims[0], nb, d->world, d->tile, part)) return rc;
+        d->peer_lo[sd] = part[2];
+        d->peer_hi[sd] = part[3];
+        for (int i = 0; i < 2; ++i) d->peerP[sd][i] = static_cast<float*>(ptr[i]);
+        // my slot in the neighbour's flag pair: I am its upper neighbour if sd == 0
+        d->peerF[sd] = static_cast<unsigned*>(ptr[2]) + (sd == 0 ? 1 : 0);
+    }
+    return STENCIL_OK;
+}
+
+extern "C" void stencil_hexdist_destroy(void* hd) {
+    auto* d = static_cast<stencil_hexdist_s*>(hd);
+    if (!d) return;
+    cudaSetDevice(d->device);
+    cudaDeviceSynchronize();
+    for (int sd = 0; sd < 2; ++sd) {
+        if (d->peerP[sd][0]) cudaIpcCloseMemHandle(d->peerP[sd][0]);
+        if (d->peerP[sd][1]) cudaIpcCloseMemHandle(d->peerP[sd][1]);
+        if (d->peerF[sd]) cudaIpcCloseMemHandle(d->peerF[sd] - (sd == 0 ? 1 : 0));
+    }
+    if (d->me.P[0]) cudaFree(d->me.P[0]);
+    if (d->me.P[1]) cudaFree(d->me.P[1]);
+    if (d->flags) cudaFree(d->flags);
+    delete d;
+}
+
+// A_T on this rank: d_in_slab / d_out_slab hold the rows [held_lo, held_hi) of
+// stencil_hexdist_partition; d_in_slab must also cover the stored rows, so the
+// caller passes the stored rows [x_lo, x_hi) of level 0 as d_in_stored.
+extern "C" int stencil_run_hexdist(stencil_t h, void* hd, const float* d_in_stored, float* d_out_slab, int64_t T,
+                                   int threads, void* cuda_stream) {
+    auto* d = static_cast<stencil_hexdist_s*>(hd);
+    if (!h || !d || !d_in_stored || !d_out_slab || T < 1) return STENCIL_EINVAL;
+    if (h->sticky) return h->sticky;
+    const stencil_tile tile = d->tile;
+    int G, thr;
+    if (int rc = check_tile(h->ndims, tile, threads, h->smem_optin, &G, &thr, h->kind)) return rc;
+    cudaStream_t s = (cudaStream_t)cuda_stream;
+    cudaSetDevice(h->device);
+    const int64_t S1 = h->dims[0], S2 = h->dims[1];
+    HexRank& r = d->me;
+    const size_t bytes = (size_t)((r.x_hi - r.x_lo) * S2) * sizeof(float);
+    for (int i = 0; i < 2; ++i) cudaMemcpyAsync(r.P[i], d_in_stored, bytes, cudaMemcpyDeviceToDevice, s);
+    if (int rc = prepare_rows(h, h->dims, T, tile, thr)) return rc;
+    hex_kernel_t kern = get_hex_kernel(h->ndims, h->kind, h->mode, h->has_c, h->defw, tile.s2);
+    const int64_t smem = smem_bytes(h->ndims, tile.t, tile.s1, tile.s2, tile.s3, h->R);
+    std::vector<RowPlan> rows;
+    plan_rows(h->ndims, h->dims, T, tile, rows, h->R);
+    HexParams p;
+    memset(&p, 0, sizeof(p));
+    p.S1 = S1; p.S2 = S2; p.S3 = 1; p.T = T;
+    p.tT = tile.t; p.tS1 = tile.s1; p.tS2 = tile.s2;
+    p.G = G; p.P = 2 * tile.s1 + tile.t; p.R = 1; p.J = 1;
+    for (int j = 0; j < kMaxPts; ++j) p.w[j] = h->w[j];
+    p.c = h->c; p.kappa = h->kappa;
+    p.in = r.Pg[0]; p.plane[0] = r.Pg[0]; p.plane[1] = r.Pg[1];
+    p.npeer = d->world > 1;
+    for (int sd = 0; sd < 2; ++sd) {
+        for (int i = 0; i < 2; ++i) p.peer[sd][i] = d->peerP[sd][i] ? d->peerP[sd][i] - d->peer_lo[sd] * S2 : nullptr;
+        p.peer_lo[sd] = d->peerP[sd][0] ? d->peer_lo[sd] : 0;
+        p.peer_hi[sd] = d->peerP[sd][0] ? d->peer_hi[sd] : 0;
+    }
+    const bool lo = d->peerF[0] != nullptr, hi = d->peerF[1] != nullptr;
+    int64_t nl = 2;
+    // Epoch handshake (monotonic counters, Nw + 1 steps per run): step 1 = "my
+    // planes hold this run's level 0" (signalled after the copies above, so a
+    // neighbour's peer stores can never be overwritten by them, and only after
+    // my previous run's output copy), step m + 1 = "my row m is done".  Row m
+    // waits for both neighbours' step m.
+    const unsigned base = d->epoch;
+    if (lo || hi) {
+        hexdist_signal_kernel<<<1, 32, 0, s>>>(d->peerF[0], d->peerF[1], base + 1);
+        ++nl;
+    }
+    unsigned m = 0;
+    for (auto& row : rows) {
+        ++m;
+        if (lo || hi) {
+            hexdist_wait_kernel<<<1, 32, 0, s>>>(d->flags, lo ? base + m : 0u, hi ? base + m : 0u);
+            ++nl;
+        }
+        p.t0 = row.t0; p.tau_lo = row.tau_lo; p.tau_hi = row.tau_hi; p.n2 = row.n2; p.n3 = 1;
+        auto first_at = [&](int64_t b) {
+            const int64_t num = 2 * b - tile.s1 - 2 * row.xbase;
+            return num <= 0 ? (int64_t)0 : cdiv(num, 2 * (int64_t)p.P);
+        };
+        const int64_t jlo = d->rank == 0 ? 0 : std::min<int64_t>(first_at(r.b0), row.w);
+        const int64_t jhi = d->rank == d->world - 1 ? row.w : std::min<int64_t>(first_at(r.b1), row.w);
+        if (jhi > jlo) {
+            p.xbase = row.xbase + jlo * p.P;
+            void* args[] = {&p};
+            cudaError_t e = cudaLaunchKernel((const void*)kern, dim3((unsigned)(jhi - jlo)), dim3(thr), args,
+                                             (size_t)smem, s);
+            if (e != cudaSuccess) return cuda_fail(h, e);
+            ++nl;
+        }
+        if (lo || hi) {
+            hexdist_signal_kernel<<<1, 32, 0, s>>>(d->peerF[0], d->peerF[1], base + m + 1);
+            ++nl;
+        }
+    }
+    d->epoch = base + m + 1;
+    const int64_t n = (r.held_hi - r.held_lo) * S2;
+    cudaMemcpyAsync(d_out_slab, r.Pg[T & 1] + r.held_lo * S2, (size_t)n * sizeof(float), cudaMemcpyDeviceToDevice, s);
+    h->last_launches = nl;
+    return cuda_fail(h, cudaGetLastError());
+}
