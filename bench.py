@@ -237,6 +237,9 @@ def main(argv=None):
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-overlap", action="store_true",
                     help="N>1: exchange, then the whole ghost-extended slab (no overlap)")
+    ap.add_argument("--exchange", default="slab", choices=["slab", "hexdist"],
+                    help="N > 1: NCCL ghost-row slabs (default) or the non-redundant hexagon-aligned decomposition "
+                         "with peer-mapped facet stores (f1, 2D configs)")
     ap.add_argument("--weak", action="store_true",
                     help="N > 1: one config-sized slab per rank (default: strong scaling, the config's grid split "
                          "over the ranks)")

@@ -91,20 +91,42 @@ def bench_main(args, cfg, cfgname, configs):
         threads = args.threads
     if getattr(args, "no_overlap", False):
         overlap = 0
-    comm = init_comm(rank, world, local, dist)
-    hhc.stencil_dist_set_overlap(comm, overlap)
-    lo, hi = slab_rows(dims[0], rank, world, tile[0])
-    host = field(CONFIG_SEEDS[cfgname], dims, row_start=lo, nrows=hi - lo)
-    d_in = torch.from_numpy(host).to(dev)
-    d_out = torch.empty_like(d_in)
     mode = hhc.FUSED if args.mode == "fused" else hhc.PLAIN
     h = hhc.stencil_create(kind, dims, mode=mode)
     stream = torch.cuda.current_stream()
     launches = [0]
+    hexdist = getattr(args, "exchange", "slab") == "hexdist"
+    if hexdist:
+        # f1: hexagons by centre column, facets peer-stored into the neighbours' planes
+        # (CUDA IPC handles carried by torch.distributed; no NCCL on the data path)
+        comm = None
+        b0, b1, xl, xh, lo, hi = hhc.stencil_hexdist_partition(dims[0], rank, world, tile)
+        obj, mine = hhc.stencil_hexdist_create(h, rank, world, tile)
+        allh = [None] * world
+        dist.all_gather_object(allh, mine)
+        hhc.stencil_hexdist_connect(h, obj, allh[rank - 1] if rank > 0 else None,
+                                    allh[rank + 1] if rank < world - 1 else None)
+        dist.barrier()
+        stored = torch.from_numpy(field(CONFIG_SEEDS[cfgname], dims, row_start=xl, nrows=xh - xl)).to(dev)
+        host = field(CONFIG_SEEDS[cfgname], dims, row_start=lo, nrows=hi - lo)
+        d_in = stored
+        d_out = torch.empty((hi - lo,) + tuple(dims[1:]), dtype=torch.float32, device=dev)
+        overlap = 0
 
-    def one():
-        hhc.stencil_run_dist(h, comm, d_in, d_out, T, tile, threads, stream)
-        launches[0] += hhc.stencil_last_launches(h)
+        def one():
+            hhc.stencil_run_hexdist(h, obj, d_in, d_out, T, threads, stream)
+            launches[0] += hhc.stencil_last_launches(h)
+    else:
+        comm = init_comm(rank, world, local, dist)
+        hhc.stencil_dist_set_overlap(comm, overlap)
+        lo, hi = slab_rows(dims[0], rank, world, tile[0])
+        host = field(CONFIG_SEEDS[cfgname], dims, row_start=lo, nrows=hi - lo)
+        d_in = torch.from_numpy(host).to(dev)
+        d_out = torch.empty_like(d_in)
+
+        def one():
+            hhc.stencil_run_dist(h, comm, d_in, d_out, T, tile, threads, stream)
+            launches[0] += hhc.stencil_last_launches(h)
 
     for _ in range(args.warmup):
         one()
@@ -136,12 +158,12 @@ def bench_main(args, cfg, cfgname, configs):
     # e2e through the public API: pinned host slab -> device, the run, the slab -> host
     e2e = None
     if not args.no_e2e:
-        h_in = torch.from_numpy(host).pin_memory()
-        h_out = torch.empty_like(h_in).pin_memory()
+        h_in = torch.from_numpy(d_in.cpu().numpy()).pin_memory()
+        h_out = torch.empty(tuple(d_out.shape), dtype=torch.float32).pin_memory()
 
         def one_e2e():
             d_in.copy_(h_in, non_blocking=True)
-            hhc.stencil_run_dist(h, comm, d_in, d_out, T, tile, threads, stream)
+            one()
             h_out.copy_(d_out, non_blocking=True)
             torch.cuda.synchronize()
 
@@ -152,10 +174,10 @@ def bench_main(args, cfg, cfgname, configs):
             one_e2e()
         et = torch.tensor([time.perf_counter() - t0], device=dev)
         dist.all_reduce(et, op=dist.ReduceOp.MAX)
-        nb = torch.tensor([float(host.nbytes)], device=dev)
+        nb = torch.tensor([float(h_in.numel() * 4), float(h_out.numel() * 4)], device=dev)
         dist.all_reduce(nb, op=dist.ReduceOp.SUM)
         e2e = {"value": hhc.updates(dims, T) * args.steps / float(et.item()) / 1e9, "unit": "GStencil-updates/s",
-               "h2d_bytes_per_step": int(nb[0].item()), "d2h_bytes_per_step": int(nb[0].item())}
+               "h2d_bytes_per_step": int(nb[0].item()), "d2h_bytes_per_step": int(nb[1].item())}
     n_upd = hhc.updates(dims, T)
     if rank == 0:
         line = {"metric": "GStencil-updates/s", "value": round(n_upd * args.steps / dt / 1e9, 3),
@@ -165,10 +187,12 @@ def bench_main(args, cfg, cfgname, configs):
                 "config": {"workload": cfgname + ": " + cfg["desc"] + (
                                "" if strong else f", weak-scaled: {world} slabs of the config's rows, global grid "
                                                  f"{'x'.join(map(str, dims))}"), "tile": list(tile), "threads": threads,
-                           "parallelism": f"{world} S1 slabs, ghost depth {tile[0]}, ncclSend/ncclRecv every time "
-                                          f"tile (stencil_run_dist, "
-                                          + ("edge sub-slabs overlapped with the interior)" if overlap
-                                             else "exchange then the ghost-extended slab)"),
+                           "parallelism": (f"{world} ranks, hexagons by centre column, facets peer-stored over "
+                                           f"NVLink into the neighbours' planes (stencil_run_hexdist, f1)" if hexdist else
+                                           f"{world} S1 slabs, ghost depth {tile[0]}, ncclSend/ncclRecv every time "
+                                           f"tile (stencil_run_dist, "
+                                           + ("edge sub-slabs overlapped with the interior)" if overlap
+                                              else "exchange then the ghost-extended slab)")),
                            "l2": "inputs larger than L2"},
                 "roofline": bench.alu_roofline(kind, n_upd * args.steps / dt / world, bench.load_peaks(),
                                                traffic=None,
@@ -179,7 +203,11 @@ def bench_main(args, cfg, cfgname, configs):
                 "e2e": e2e, "clocks": clocks, "gpu_launches": n_launch}
         print(json.dumps(line))
     torch.cuda.synchronize()
+    dist.barrier()
+    if hexdist:
+        hhc.stencil_hexdist_destroy(obj)
+    else:
+        hhc.stencil_dist_destroy(comm)
     hhc.stencil_destroy(h)
-    hhc.stencil_dist_destroy(comm)
     dist.destroy_process_group()
     return 0

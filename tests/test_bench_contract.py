@@ -54,3 +54,11 @@ def test_torchrun_slab_path_world1():
     for k in KEYS + ["roofline", "e2e", "clocks", "gpu_launches"]:
         assert k in d, k
     assert d["n_gpus"] == 1 and d["value"] > 0 and d["gpu_launches"] > 0
+
+
+@pytest.mark.gpu
+def test_torchrun_hexdist_path_world1():
+    d = _run(["-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "1", "--master-addr", "127.0.0.1",
+              "--master-port", "29534", "bench.py", "--gpus", "2", "--config", "C1", "--exchange", "hexdist",
+              "--steps", "2", "--warmup", "3"])
+    assert d["n_gpus"] == 1 and d["value"] > 0 and "f1" in d["config"]["parallelism"]
