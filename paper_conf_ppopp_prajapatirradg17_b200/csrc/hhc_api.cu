@@ -1053,6 +1053,12 @@ extern "C" int stencil_run_hexdist(stencil_t h, void* hd, const float* d_in_stor
         }
     }
     d->epoch = base + m + 1;
+    // the neighbours' last row may still store level-T facets of my rows: wait for it
+    // before the output copy (and before the next run's level-0 copies)
+    if (lo || hi) {
+        hexdist_wait_kernel<<<1, 32, 0, s>>>(d->flags, lo ? base + m + 1 : 0u, hi ? base + m + 1 : 0u);
+        ++nl;
+    }
     const int64_t n = (r.held_hi - r.held_lo) * S2;
     cudaMemcpyAsync(d_out_slab, r.Pg[T & 1] + r.held_lo * S2, (size_t)n * sizeof(float), cudaMemcpyDeviceToDevice, s);
     h->last_launches = nl;
