@@ -85,6 +85,8 @@ struct stencil_s {
     float* scratch = nullptr;
     unsigned* flags = nullptr;
     int64_t flags_n = 0;
+    float* faceg = nullptr;     // 2D J > 1: face scratch [w][n2][tT][NX][2]
+    int64_t faceg_n = 0;
     float* h_in_dev = nullptr;   // stencil_run_host device buffers
     float* h_out_dev = nullptr;
     int sticky = 0;
@@ -206,6 +208,7 @@ extern "C" void stencil_destroy(stencil_t h) {
     drop_graphs(h);
     if (h->scratch) cudaFree(h->scratch);
     if (h->flags) cudaFree(h->flags);
+    if (h->faceg) cudaFree(h->faceg);
     if (h->h_in_dev) cudaFree(h->h_in_dev);
     if (h->h_out_dev) cudaFree(h->h_out_dev);
     if (h->cap_stream) cudaStreamDestroy(h->cap_stream);
@@ -350,15 +353,20 @@ static int choose_J(stencil_t h, const RowPlan& r) {
     return J;
 }
 
+// 2D rows get J > 1 blocks per hexagon only in planes mode (slab sub-problems of the
+// multi-GPU path, where few hexagons share the GPU); full-grid runs keep J = 1.
+static bool j_rows(const stencil_t h, bool planes) { return h->ndims == 3 || (h->ndims == 2 && planes); }
+
 // Everything that must not happen inside stream capture: the kernel's smem
-// attribute, its occupancy (for J), and the 3D flag buffer.
-static int prepare_rows(stencil_t h, const int64_t* dims, int64_t T, stencil_tile tile, int thr) {
+// attribute, its occupancy (for J), the flag buffer and the 2D face scratch.
+static int prepare_rows(stencil_t h, const int64_t* dims, int64_t T, stencil_tile tile, int thr,
+                        bool planes = false) {
     hex_kernel_t k = get_hex_kernel(h->ndims, h->kind, h->mode, h->has_c, h->defw, tile.s2);
     if (!k) return STENCIL_EINVAL;
     const int64_t smem = smem_bytes(h->ndims, tile.t, tile.s1, tile.s2, tile.s3, h->R);
     cudaError_t e = cudaFuncSetAttribute((const void*)k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return cuda_fail(h, e);
-    if (h->ndims != 3) return STENCIL_OK;
+    if (!j_rows(h, planes)) return STENCIL_OK;
     int occ = 1;
     e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, (const void*)k, thr, (size_t)smem);
     if (e != cudaSuccess) return cuda_fail(h, e);
@@ -369,6 +377,18 @@ static int prepare_rows(stencil_t h, const int64_t* dims, int64_t T, stencil_til
     for (auto& r : rows) {
         const int J = choose_J(h, r);
         if (J > 1) need = std::max<int64_t>(need, (int64_t)r.w * r.n2);
+    }
+    if (h->ndims == 2 && need > 0) {
+        const int64_t fneed = need * tile.t * (int64_t)(tile.s1 + tile.t + 2) * 2;
+        if (fneed > h->faceg_n) {
+            drop_graphs(h);
+            if (h->faceg) cudaFree(h->faceg);
+            h->faceg = nullptr;
+            h->faceg_n = 0;
+            e = cudaMalloc(&h->faceg, fneed * sizeof(float));
+            if (e != cudaSuccess) return cuda_fail(h, e);
+            h->faceg_n = fneed;
+        }
     }
     if (need > h->flags_n) {
         // the cached graphs captured the old flag pointer (memset node and kernel
@@ -389,7 +409,7 @@ static int prepare_rows(stencil_t h, const int64_t* dims, int64_t T, stencil_til
 // result (level T) lands in plane[T & 1].  Ring values are read from `ring`.
 static int enqueue_rows(stencil_t h, const int64_t* dims, const float* ring, float* plane0, float* plane1,
                         int64_t T, stencil_tile tile, int G, int thr, cudaStream_t s, int64_t* launches,
-                        std::vector<cudaEvent_t>* evs = nullptr) {
+                        std::vector<cudaEvent_t>* evs = nullptr, bool planes = false) {
     std::vector<RowPlan> rows;
     plan_rows(h->ndims, dims, T, tile, rows, h->R);
     hex_kernel_t k = get_hex_kernel(h->ndims, h->kind, h->mode, h->has_c, h->defw, tile.s2);
@@ -400,7 +420,7 @@ static int enqueue_rows(stencil_t h, const int64_t* dims, const float* ring, flo
     // 3D: thread blocks per slab J (pipelined along S2, flags in global memory);
     // all blocks of a launch must be co-resident when J > 1 (no deadlock).
     // Occupancy and the flag buffer come from prepare_rows (outside capture).
-    if (h->ndims == 3) {
+    if (j_rows(h, planes)) {
         int64_t need = 0;
         for (auto& r : rows) {
             r.J = choose_J(h, r);
@@ -427,6 +447,7 @@ static int enqueue_rows(stencil_t h, const int64_t* dims, const float* ring, flo
     p.c = h->c;
     p.kappa = h->kappa;
     p.flags = h->flags;
+    p.faceg = h->faceg;
     p.compute_only = h->compute_only;
     for (auto& r : rows) {
         p.t0 = r.t0; p.xbase = r.xbase; p.tau_lo = r.tau_lo; p.tau_hi = r.tau_hi;
@@ -468,7 +489,7 @@ static int enqueue_spec(stencil_t h, const RunSpec& r, cudaStream_t s, int64_t* 
     } else {
         float* p0 = const_cast<float*>(r.a);
         launch_copy_ring(p0, r.b, r.dims[0], r.dims[1], r.dims[2], s, h->R); ++nl;
-        rc = enqueue_rows(h, r.dims, p0, p0, r.b, r.T, r.tile, r.G, r.thr, s, &nrows, nullptr);
+        rc = enqueue_rows(h, r.dims, p0, p0, r.b, r.T, r.tile, r.G, r.thr, s, &nrows, nullptr, true);
     }
     *launches = nl + nrows;
     return rc;
@@ -483,7 +504,7 @@ static bool same_spec(const RunSpec& x, const RunSpec& y) {
 
 // Run a spec through the CUDA-graph cache (captured once per spec, replayed).
 static int run_spec(stencil_t h, const RunSpec& r, cudaStream_t s) {
-    int prc = r.planes_mode == 2 ? STENCIL_OK : prepare_rows(h, r.dims, r.T, r.tile, r.thr);
+    int prc = r.planes_mode == 2 ? STENCIL_OK : prepare_rows(h, r.dims, r.T, r.tile, r.thr, r.planes_mode == 1);
     if (prc) return prc;
     const bool use_graph = getenv("HHC_NO_GRAPH") == nullptr && !h->compute_only;
     if (!use_graph) {

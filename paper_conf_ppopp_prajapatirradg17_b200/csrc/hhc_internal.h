@@ -28,6 +28,7 @@ struct HexParams {
     int J;                  // 3D: thread blocks per hexagonal slab (pipelined along S2)
     unsigned* flags;        // 3D, J > 1: progress flags [w][n2]
     unsigned epoch;         // flag value base for this row
+    float* faceg;           // 2D, J > 1: face scratch [w][n2][tT][NX][2]
     float w[kMaxPts];       // weights in canonical order (reading R4)
     float c;                // Eq. 1 constant
     float kappa;            // Gradient-2D

@@ -190,6 +190,31 @@ def test_hexdist_local_virtual_ranks(kind, dims, T, tile, world, threads):
         assert n > 0
 
 
+@pytest.mark.parametrize("kind,dims,T,tile,threads", [
+    (hhc.HEAT2D_9PT, (200, 2000), 37, (8, 6, 64), 0),
+    (hhc.GRADIENT2D, (90, 3000), 21, (16, 8, 128), 64),
+    (hhc.JACOBI2D_5PT, (70, 5000), 50, (32, 12, 512), 384),
+])
+def test_planes_2d_pipelined_blocks(kind, dims, T, tile, threads):
+    """stencil_run_planes (the slab sub-problem) on a short, wide 2D domain: few
+    hexagons, so each prism is split over J > 1 blocks pipelined along S2, the
+    2-column face of sub-tile j2-1 handed over through global scratch after an
+    acquire on its flag.  Must equal the oracle on the same domain (its outer
+    rows are the fixed ring)."""
+    for mode in (hhc.PLAIN, hhc.FUSED):
+        a = field(500 + kind + mode, dims)
+        s = hhc.stencil_create(kind, dims, mode=mode)
+        p0 = torch.from_numpy(a).to(DEV)
+        p1 = torch.empty_like(p0)
+        for rep in range(2):                      # graph replay with the flags reset per run
+            p0.copy_(torch.from_numpy(a).to(DEV))
+            hhc.stencil_run_planes(s, dims[0], p0, p1, T, tile, threads)
+            torch.cuda.synchronize()
+            got = (p0 if T % 2 == 0 else p1).cpu().numpy()
+            assert_bits(got, oracle.run(kind, a, T, mode), f"planes J>1 kind {kind} mode {mode} rep {rep}")
+        hhc.stencil_destroy(s)
+
+
 def test_dist_world1_nccl_free():
     """stencil_run_dist on a world-1 communicator (no NCCL needed): the slab is
     the whole grid."""
