@@ -20,6 +20,9 @@ inline int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
 // Stencil radius of the kind being modelled (1; 2-4 for the f4 kinds, reading F4:
 // slopes, pitch, footprints and facets scale by R), set by model_predict.
 thread_local int64_t g_R = 1;
+// Reading M8 for 2D: set while M7 evaluates a slab sub-problem -- the library runs
+// those in planes mode, where a 2D hexagonal prism is split over J pipelined blocks.
+thread_local bool g_planes = false;
 
 int ndims_of(int kind) {
     switch (kind) {
@@ -173,7 +176,17 @@ double talg_exact(int nd, const int64_t* S, int64_t T, const stencil_tile& tl, c
             mi = (double)reads;
             mo = (double)writes;
         } else if (nd == 2) {
-            Nsub = (double)cdiv(S2 + nlev - 1, tS2);
+            const int64_t n2 = cdiv(S2 + nlev - 1, tS2);
+            Nsub = (double)n2;
+            if (g_planes) {
+                // M8 in 2D (slab sub-problems): J blocks per prism, the face (2 columns per
+                // row and level) written and read back through global memory
+                J = std::max<int64_t>(1, std::min<int64_t>(n2, ((int64_t)hw.n_sm * k) / w));
+                if (J > 1) {
+                    Nsub = (double)(cdiv(n2, J) + (J - 1));
+                    extra = 4.0 * (double)area;
+                }
+            }
             mi = (double)reads * (double)(tS2 + 2);
             mo = (double)writes * (double)tS2;
         } else {
@@ -219,7 +232,10 @@ double talg_dist(int nd, const int64_t* S, int64_t T, const stencil_tile& tl, co
     const double t_exch = (double)g * plane / bw + hw.link_latency_s;
     auto run = [&](int64_t rows, int64_t Tt) {
         const int64_t Sl[3] = {rows, S[1], nd == 3 ? S[2] : 1};
-        return f(nd, Sl, Tt, tl, hw);
+        g_planes = true;
+        const double v = f(nd, Sl, Tt, tl, hw);
+        g_planes = false;
+        return v;
     };
     const int64_t n = cdiv(T, tl.t);
     const int64_t Tlast = T - (n - 1) * tl.t;

@@ -171,7 +171,7 @@ def test_multi_gpu_model_hand_example():
     inner S2 = 100 -> T_exch = 8*100*4 B / 1e9 B/s + 1e-6 = 4.2e-6 s."""
     calls = []
 
-    def fake(nd, S, T, tile, hw):
+    def fake(nd, S, T, tile, hw, R=1, planes=False):
         calls.append((S[0], T))
         return 1e-6 * S[0] * T                       # 1 us per row-step
 
