@@ -59,7 +59,7 @@ def max_rel(got, ref):
 
 
 TILES_2D = [(2, 1, 32), (4, 3, 32), (8, 5, 64), (6, 2, 32), (10, 7, 96), (16, 4, 128), (2, 9, 64)]
-TILES_3D = [(2, 1, 1, 32), (4, 2, 3, 32), (6, 3, 4, 64), (8, 2, 2, 32), (2, 5, 6, 32)]
+TILES_3D = [(2, 1, 1, 32), (4, 2, 3, 32), (6, 3, 4, 64), (8, 2, 2, 32), (2, 5, 6, 32), (4, 3, 2, 96), (6, 2, 3, 128)]
 
 
 @pytest.mark.parametrize("kind", [hhc.JACOBI2D_5PT, hhc.HEAT2D_9PT, hhc.GRADIENT2D, hhc.LAPLACIAN2D_5PT])
@@ -92,11 +92,19 @@ def test_parity_3d_small(kind, mode):
 
 @pytest.mark.parametrize("threads", [0, 8, 16, 24, 64])
 def test_threads_variants(threads):
+    """K1 with 1-8 x-groups; K2 (3D) likewise on a grid whose rows are 16-B chunks."""
     a = field(5, (77, 133))
     tile = (6, 3, 32)
     exp = oracle.run(hhc.HEAT2D_9PT, a, 19, hhc.FUSED)
     got = gpu_run(hhc.HEAT2D_9PT, a, 19, tile, hhc.FUSED, threads=threads)
     assert_bits(got, exp, f"threads {threads}")
+    b = field(15, (37, 29, 68))
+    exp3 = oracle.run(hhc.HEAT3D_7PT, b, 17, hhc.FUSED)
+    for tile3 in ((6, 3, 2, 32), (4, 5, 3, 64)):
+        base = (tile3[3] // 4) * tile3[2]             # K2 column threads: 4 tS3 columns per tS2 line
+        thr = base * max(1, threads // 8)
+        if thr <= 512:
+            assert_bits(gpu_run(hhc.HEAT3D_7PT, b, 17, tile3, hhc.FUSED, threads=thr), exp3, f"3D threads {thr}")
 
 
 def test_T0_and_tiny_grids():
@@ -128,6 +136,8 @@ def test_custom_coefficients_and_c():
     (hhc.GRADIENT2D, (700, 900), 40, (8, 6, 256)),
     (hhc.HEAT3D_7PT, (64, 66, 130), 20, (8, 4, 4, 32)),
     (hhc.LAPLACIAN3D_27PT, (60, 50, 70), 12, (4, 3, 4, 64)),
+    (hhc.HEAT3D_7PT, (50, 60, 136), 21, (6, 4, 5, 64)),            # S3 % 4 == 0: 16-B u2-halo loads
+    (hhc.LAPLACIAN3D_27PT, (41, 37, 200), 13, (8, 3, 4, 128)),
 ])
 def test_parity_mid_size(kind, dims, T, tile):
     a = field(42, dims)
