@@ -263,7 +263,7 @@ extern "C" int stencil_tile_resources(stencil_kind kind, int ndims, stencil_tile
         // Eq. 11's register bound (reading M4): the kernel the library launches for this
         // (kind, mode, tile) with default weights, from cudaFuncGetAttributes; 0 if kind is 0
         // or no device is visible (the attribute query needs a CUDA context)
-        *regs = kind != 0 ? hex_kernel_regs(ndims, kind, mode, false, true, tile.s2) : 0;
+        *regs = kind != 0 ? hex_kernel_regs(ndims, kind, mode, false, true, tile.s2, tile.s3) : 0;
         cudaGetLastError();
     }
     return STENCIL_OK;
@@ -275,7 +275,7 @@ extern "C" int stencil_tile_occupancy(stencil_kind kind, int ndims, stencil_tile
     int G, thr;
     const int rc = check_tile(ndims, tile, threads, 227 * 1024, &G, &thr, kind);
     if (rc) return rc;
-    hex_kernel_t k = get_hex_kernel(ndims, kind, mode, false, true, tile.s2);
+    hex_kernel_t k = get_hex_kernel(ndims, kind, mode, false, true, tile.s2, tile.s3);
     if (!k) return STENCIL_EINVAL;
     const int64_t smem = smem_bytes(ndims, tile.t, tile.s1, tile.s2, tile.s3, kind_radius(kind));
     cudaError_t e = cudaFuncSetAttribute((const void*)k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
@@ -361,7 +361,7 @@ static bool j_rows(const stencil_t h, bool planes) { return h->ndims == 3 || (h-
 // attribute, its occupancy (for J), the flag buffer and the 2D face scratch.
 static int prepare_rows(stencil_t h, const int64_t* dims, int64_t T, stencil_tile tile, int thr,
                         bool planes = false) {
-    hex_kernel_t k = get_hex_kernel(h->ndims, h->kind, h->mode, h->has_c, h->defw, tile.s2);
+    hex_kernel_t k = get_hex_kernel(h->ndims, h->kind, h->mode, h->has_c, h->defw, tile.s2, h->ndims == 3 ? tile.s3 : 0);
     if (!k) return STENCIL_EINVAL;
     const int64_t smem = smem_bytes(h->ndims, tile.t, tile.s1, tile.s2, tile.s3, h->R);
     cudaError_t e = cudaFuncSetAttribute((const void*)k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
@@ -412,7 +412,7 @@ static int enqueue_rows(stencil_t h, const int64_t* dims, const float* ring, flo
                         std::vector<cudaEvent_t>* evs = nullptr, bool planes = false) {
     std::vector<RowPlan> rows;
     plan_rows(h->ndims, dims, T, tile, rows, h->R);
-    hex_kernel_t k = get_hex_kernel(h->ndims, h->kind, h->mode, h->has_c, h->defw, tile.s2);
+    hex_kernel_t k = get_hex_kernel(h->ndims, h->kind, h->mode, h->has_c, h->defw, tile.s2, h->ndims == 3 ? tile.s3 : 0);
     if (!k) return STENCIL_EINVAL;
     const int64_t smem = smem_bytes(h->ndims, tile.t, tile.s1, tile.s2, tile.s3, h->R);
     int64_t nl = 0;
@@ -831,7 +831,7 @@ extern "C" int stencil_run_hexdist_local(stencil_t h, int world, const float* d_
         }
     }
     if (int rc = prepare_rows(h, h->dims, T, tile, thr)) { release(); return rc; }
-    hex_kernel_t kern = get_hex_kernel(h->ndims, h->kind, h->mode, h->has_c, h->defw, tile.s2);
+    hex_kernel_t kern = get_hex_kernel(h->ndims, h->kind, h->mode, h->has_c, h->defw, tile.s2, h->ndims == 3 ? tile.s3 : 0);
     const int64_t smem = smem_bytes(h->ndims, tile.t, tile.s1, tile.s2, tile.s3, h->R);
     std::vector<RowPlan> rows;
     plan_rows(h->ndims, h->dims, T, tile, rows, h->R);
@@ -1016,7 +1016,7 @@ extern "C" int stencil_run_hexdist(stencil_t h, void* hd, const float* d_in_stor
     const size_t bytes = (size_t)((r.x_hi - r.x_lo) * S2) * sizeof(float);
     for (int i = 0; i < 2; ++i) cudaMemcpyAsync(r.P[i], d_in_stored, bytes, cudaMemcpyDeviceToDevice, s);
     if (int rc = prepare_rows(h, h->dims, T, tile, thr)) return rc;
-    hex_kernel_t kern = get_hex_kernel(h->ndims, h->kind, h->mode, h->has_c, h->defw, tile.s2);
+    hex_kernel_t kern = get_hex_kernel(h->ndims, h->kind, h->mode, h->has_c, h->defw, tile.s2, h->ndims == 3 ? tile.s3 : 0);
     const int64_t smem = smem_bytes(h->ndims, tile.t, tile.s1, tile.s2, tile.s3, h->R);
     std::vector<RowPlan> rows;
     plan_rows(h->ndims, h->dims, T, tile, rows, h->R);

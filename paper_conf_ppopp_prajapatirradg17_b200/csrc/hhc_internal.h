@@ -76,8 +76,8 @@ inline int column_threads(int ndims, int tS2, int tS3) {
 }
 
 typedef void (*hex_kernel_t)(HexParams);
-hex_kernel_t get_hex_kernel(int ndims, int kind, int mode, bool has_c, bool defw, int s2);
-int hex_kernel_regs(int ndims, int kind, int mode, bool has_c, bool defw, int s2);
+hex_kernel_t get_hex_kernel(int ndims, int kind, int mode, bool has_c, bool defw, int s2, int s3 = 0);
+int hex_kernel_regs(int ndims, int kind, int mode, bool has_c, bool defw, int s2, int s3 = 0);
 void launch_copy_ring(const float* in, float* out, int64_t S1, int64_t S2, int64_t S3, void* stream, int R = 1);
 void launch_copy_full(const float* in, float* out, int64_t n, void* stream);
 
