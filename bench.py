@@ -35,11 +35,16 @@ CONFIGS = {
                desc="Jacobi-2D 5-point fp32, 256x256, T=64"),
     "C2": dict(kind=2, dims=(8192, 8192), T=1024, tile=(32, 12, 512, 0), threads=384,
                desc="Heat-2D 9-point fp32, 8192x8192, T=1024"),
+    # tiles_by_gpus: the tile per GPU count under torchrun, the best measured on one GPU for
+    # the slab each rank holds (scripts/slab_tiles.py -> profiles/r02/slab_C{3,4,5}.json)
     "C3": dict(kind=3, dims=(16384, 16384), T=512, tile=(32, 12, 512, 0), threads=384,
+               tiles_by_gpus={2: (32, 12, 512, 0), 4: (24, 4, 512, 0), 8: (16, 4, 512, 0)},
                desc="Gradient-2D fp32, 16384x16384, T=512"),
     "C4": dict(kind=4, dims=(512, 512, 512), T=256, tile=(8, 8, 16, 64), threads=512,
+               tiles_by_gpus={2: (8, 6, 16, 64), 4: (8, 2, 16, 64), 8: (6, 2, 16, 64)},
                desc="Heat-3D 7-point fp32, 512^3, T=256"),
     "C5": dict(kind=5, dims=(768, 768, 768), T=128, tile=(8, 6, 8, 64), threads=256,
+               tiles_by_gpus={8: (8, 2, 16, 64)}, threads_by_gpus={8: 512},
                desc="Laplacian-3D 27-point fp32, 768^3, T=128"),
     # SURVEY §8(f) f2 (not a BASELINE.json config): the paper's 1D derivation case
     "X1": dict(kind=7, dims=(1 << 26,), T=1024, tile=(128, 2048), threads=256,

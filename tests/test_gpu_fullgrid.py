@@ -138,3 +138,26 @@ def test_affine_fixed_point_bench_launch(cfg):
     for d, k in zip(range(nd), (1.0, 2.0, 3.0)):
         aff += (k * np.arange(dims[d], dtype=np.float32)).reshape([-1 if e == d else 1 for e in range(nd)])
     assert np.array_equal(gpu_run(kind, aff, T, tile, threads), aff), cfg
+
+
+@pytest.mark.parametrize("cfg,n", [("C3", 2), ("C3", 4), ("C3", 8), ("C4", 2), ("C4", 4), ("C4", 8), ("C5", 8)])
+def test_dist_bench_tiles_virtual_ranks(cfg, n):
+    """The tile and threads bench.py uses under torchrun at n GPUs (tiles_by_gpus),
+    through the library's slab path with n virtual ranks of this GPU
+    (stencil_run_dist_local: the per-rank phases of stencil_run_dist, device copies
+    in place of NCCL) on a reduced grid with the same per-rank row count ratio:
+    every held row bit-exact against the oracle."""
+    import paper_conf_ppopp_prajapatirradg17_b200.dist as dist
+    c = bench.CONFIGS[cfg]
+    tile, threads, overlap = dist.choose_tile(c, n)
+    kind = c["kind"]
+    rows = max(3 * tile[0], 24) * n + 2
+    dims = (rows, 1100) if len(c["dims"]) == 2 else (rows, 40, 140)
+    T = 3 * tile[0] + 5
+    a = field(CONFIG_SEEDS[cfg] + 200 + n, dims)
+    s = hhc.stencil_create(kind, dims)
+    d_in = torch.from_numpy(a).to(DEV)
+    d_out = torch.full_like(d_in, float("nan"))
+    hhc.stencil_run_dist_local(s, n, d_in, d_out, T, tile, threads, overlap)
+    hhc.stencil_destroy(s)
+    assert_bits(d_out.cpu().numpy(), oracle.run(kind, a, T, hhc.FUSED), f"{cfg} n={n} tile {tile} x {threads}")
