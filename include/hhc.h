@@ -90,7 +90,9 @@ typedef struct {
     double  T_sync_s;          /* T_sync, one host-GPU synchronisation / launch (s)     */
     double  C_iter_s;          /* C_iter, one loop-body iteration per vector unit (s)   */
     int32_t regs_per_thread;   /* 0 = unknown (paper); >0 bounds k in EXACT (Eq. 11)    */
-    int32_t geometry;          /* 0 = PAPER-literal equations, 1 = EXACT (M1) */
+    int32_t geometry;          /* 0 = PAPER-literal equations, 1 = EXACT (M1),
+                                  2 = EXACT_G (+ x-group rows, M9), 3 = EXACT_GW (M9 +
+                                  the x-groups' window prologue rows, M10)              */
     int32_t threads;           /* threads per block for EXACT k; 0 = library rule      */
     int32_t max_threads_sm;    /* resident threads per SM (EXACT k); 0 = 2048           */
     int32_t n_gpus;            /* >1: slab decomposition model (M7)           */
@@ -98,6 +100,10 @@ typedef struct {
     double  link_latency_s;    /* per-message latency                                   */
     int32_t dist_overlap;      /* M7: 0 = exchange then the ghost-extended slab, 1 =
                                   edge sub-slabs overlapped with the interior           */
+    double  window_rows;       /* geometry 3 (EXACT_GW, reading M10): row
+                                  equivalents each x-group spends per level on its
+                                  register window's prologue rows (fitted with C_iter
+                                  and tau on the calibration instances); 0 elsewhere    */
 } model_hw_params;
 
 typedef struct stencil_s* stencil_t;     /* opaque; owned by the library */

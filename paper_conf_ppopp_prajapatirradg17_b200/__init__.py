@@ -28,7 +28,7 @@ KIND_NAMES = {1: "Jacobi-2D 5-point", 2: "Heat-2D 9-point", 3: "Gradient-2D", 4:
 KIND_NDIMS = {1: 2, 2: 2, 3: 2, 4: 3, 5: 3, 6: 2, 7: 1, 8: 1, 9: 1, 10: 1}
 KIND_RADIUS = {8: 2, 9: 3, 10: 4}
 PLAIN, FUSED = 0, 1
-PAPER, EXACT, EXACT_G = 0, 1, 2   # EXACT_G: EXACT + x-group rows (DESIGN reading M9)
+PAPER, EXACT, EXACT_G, EXACT_GW = 0, 1, 2, 3   # EXACT_G: + x-group rows (M9); EXACT_GW: + window rows (M10)
 
 OK, EINVAL, ETILE, ENOMEM, ECUDA, ENCCL, ENODEV = 0, -1, -2, -3, -4, -5, -6
 
@@ -57,7 +57,8 @@ class model_hw_params(ctypes.Structure):
                 ("regs_per_thread", ctypes.c_int32), ("geometry", ctypes.c_int32),
                 ("threads", ctypes.c_int32), ("max_threads_sm", ctypes.c_int32),
                 ("n_gpus", ctypes.c_int32), ("link_bytes_per_s", ctypes.c_double),
-                ("link_latency_s", ctypes.c_double), ("dist_overlap", ctypes.c_int32)]
+                ("link_latency_s", ctypes.c_double), ("dist_overlap", ctypes.c_int32),
+                ("window_rows", ctypes.c_double)]
 
 
 def make_tile(t) -> stencil_tile:

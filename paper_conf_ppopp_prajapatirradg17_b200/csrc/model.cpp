@@ -166,8 +166,11 @@ double talg_exact(int nd, const int64_t* S, int64_t T, const stencil_tile& tl, c
             else if (tau + 1 > h) writes += 4 * R;
             // reading M9 (geometry 2): the G x-groups split the row, so a level lasts
             // G*ceil(W/G) rows' worth of the block's vector units
-            const int64_t We = (hw.geometry == 2 && G > 1) ? G * cdiv(W, G) : W;
+            const int64_t We = (hw.geometry >= 2 && G > 1) ? G * cdiv(W, G) : W;
             csum += (double)cdiv(We * inner, hw.n_v);          // Eq. 15 / 27, row by row
+            // reading M10 (geometry 3): each x-group's register window first loads the
+            // rows below and at its segment -- window_rows row equivalents per group
+            if (hw.geometry == 3 && nd >= 2) csum += hw.window_rows * (double)(G * inner) / (double)hw.n_v;
         }
         double Nsub, mi, mo, extra = 0.0;
         int64_t J = 1;

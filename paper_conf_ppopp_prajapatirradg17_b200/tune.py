@@ -77,6 +77,11 @@ def b200_hw(cal: dict | None, kind: int, geometry: int, threads: int = 0,
         if geometry == hhc.EXACT_G and fitg:
             hw.C_iter_s = fitg["C_iter_s"]
             hw.tau_sync_s = fitg["tau_level_s"]
+        fitw = (cal.get("exactgw_fit") or {}).get(str(kind))
+        if geometry == hhc.EXACT_GW and fitw:
+            hw.C_iter_s = fitw["C_iter_s"]
+            hw.tau_sync_s = fitw["tau_level_s"]
+            hw.window_rows = fitw["window_rows"]
         lf = (cal.get("exact_leff") or {}).get(str(kind))
         if leff and geometry == hhc.EXACT and lf:
             hw.L_s_per_word = lf["L_s_per_word"]
@@ -169,7 +174,7 @@ def calibrate(args):
         out["T_sync_s"] = hhc.stencil_microbench(2)
         out["regs_per_thread"] = {str(k): kernel_regs(k) for k in KINDS}
     rnd = random.Random(2017)
-    citer, samples, fits, fitsg, insts, raw, full, full_all = {}, {}, {}, {}, [], {}, [], {}
+    citer, samples, fits, fitsg, fitsw, insts, raw, full, full_all = {}, {}, {}, {}, {}, [], {}, [], {}
     for kind in kinds:
         nd = hhc.KIND_NDIMS[kind]
         vals = []
@@ -202,6 +207,7 @@ def calibrate(args):
         samples[str(kind)] = {"n": len(vals), "min": min(vals), "max": max(vals)}
         fits[str(kind)] = fit_exact(kind, insts)
         fitsg[str(kind)] = fit_exact(kind, insts, hhc.EXACT_G)
+        fitsw[str(kind)] = fit_exact(kind, insts, hhc.EXACT_GW)
         full_all[str(kind)] = list(full)
         raw[str(kind)] = [[list(d), T_, list(t), v] for d, T_, t, v in insts]
         insts.clear()
@@ -210,7 +216,7 @@ def calibrate(args):
               f"EXACT fit {fits[str(kind)]}", flush=True)
     if base is not None:
         for key, new in (("C_iter_s", citer), ("C_iter_samples", samples), ("exact_fit", fits),
-                         ("exactg_fit", fitsg), ("instances", raw)):
+                         ("exactg_fit", fitsg), ("exactgw_fit", fitsw), ("instances", raw)):
             merged = dict(base.get(key) or {})
             merged.update(new)
             out[key] = merged
@@ -221,6 +227,7 @@ def calibrate(args):
         out["C_iter_samples"] = samples
         out["exact_fit"] = fits
         out["exactg_fit"] = fitsg
+        out["exactgw_fit"] = fitsw
         out["instances"] = raw          # (dims, T, tile, compute-only seconds): refits need no GPU
         out["exact_leff"], out["instances_full"] = {}, {}
     out["exact_leff"].update({k: fit_leff(out, int(k), v) for k, v in full_all.items()})
@@ -231,40 +238,71 @@ def calibrate(args):
     print(json.dumps({k: v for k, v in out.items() if k not in ("C_iter_samples", "instances", "instances_full")}))
 
 
-def _basis(kind, dims, T, tile, c_iter, tau, geometry=None):
-    """Talg_EXACT (or EXACT_G) with only C_iter / tau_sync nonzero (L = T_sync = 0)."""
+def _basis(kind, dims, T, tile, c_iter, tau, geometry=None, window=0.0):
+    """Talg_EXACT (or EXACT_G / EXACT_GW) with only C_iter / tau_sync (/ window_rows) nonzero."""
     hw = b200_hw(None, kind, hhc.EXACT if geometry is None else geometry)
     hw.C_iter_s, hw.tau_sync_s, hw.L_s_per_word, hw.T_sync_s = c_iter, tau, 0.0, 0.0
+    hw.window_rows = window
     return hhc.model_predict(kind, dims, T, tile, hw)
 
 
+def _micro_count(kind, dims, T, tile):
+    """The iteration count stencil_microbench(3) divides the compute-only time by:
+    Talg_EXACT with C_iter = 1, L = tau = T_sync = 0, the library's threads and no
+    register bound (microbench.cu), so a recorded C_iter sample v gives back the
+    measured compute-only time as v * count."""
+    hw = b200_hw(None, kind, hhc.EXACT)
+    hw.C_iter_s, hw.tau_sync_s, hw.L_s_per_word, hw.T_sync_s = 1.0, 0.0, 0.0, 0.0
+    hw.regs_per_thread = 0
+    return hhc.model_predict(kind, dims, T, tile, hw)
+
+
+def _lsq(rows):
+    """Non-negative relative least squares: rows of (basis_1/t, ..., basis_n/t) ~ 1."""
+    import numpy as np
+    A = np.array(rows, dtype=float)
+    n = A.shape[1]
+    best = None
+    for mask in range(1, 1 << n):                      # all supports; keep the best feasible one
+        cols = [j for j in range(n) if mask >> j & 1]
+        x, *_ = np.linalg.lstsq(A[:, cols], np.ones(len(A)), rcond=None)
+        if (x < 0).any():
+            continue
+        full = np.zeros(n)
+        full[cols] = x
+        err = float(np.sqrt(np.mean((A @ full - 1.0) ** 2)))
+        if best is None or err < best[1]:
+            best = (full, err)
+    return best
+
+
 def fit_exact(kind, insts, geometry=None):
-    """Reading Q14 (EXACT): the compute-only times T_i of the calibration
-    instances are fitted jointly as C_iter * A_i + tau * B_i, A_i / B_i the
-    EXACT model with only C_iter / only tau_sync set to 1 (the model is linear
-    in both when L = T_sync = 0), minimising the relative error.  tau then
-    carries the implemented kernel's real per-level cost (barrier + window
-    prologue), not a bare __syncthreads; PAPER mode keeps the paper's procedure
-    (C_iter averaged, tau_sync from its own micro-benchmark)."""
+    """Reading Q14 (EXACT, EXACT_G; M10 for EXACT_GW): the compute-only times T_i of
+    the calibration instances (T_i = the recorded C_iter sample x the micro-benchmark's
+    own EXACT iteration count) are fitted jointly as C_iter * A_i + tau * B_i
+    (+ C_iter * window_rows * P_i), A_i / B_i / P_i the model of that geometry with
+    only C_iter / only tau_sync / only the window term set, minimising the relative
+    error (non-negative).  tau then carries the implemented kernel's per-level cost
+    (barrier and the rest), not a bare __syncthreads; PAPER mode keeps the paper's
+    procedure (C_iter averaged, tau_sync from its own micro-benchmark)."""
+    g = hhc.EXACT if geometry is None else geometry
     rows = []
     for dims, T, tile, v in insts:
-        a = _basis(kind, dims, T, tile, 1.0, 0.0, geometry)
-        b = _basis(kind, dims, T, tile, 0.0, 1.0, geometry)
-        t = v * a                                    # microbench returns T_i / A_i
-        if all(math.isfinite(x) and x > 0 for x in (a, b, t)):
-            rows.append((a / t, b / t))
-    if len(rows) < 2:
+        t = v * _micro_count(kind, dims, T, tile)
+        a = _basis(kind, dims, T, tile, 1.0, 0.0, g)
+        b = _basis(kind, dims, T, tile, 0.0, 1.0, g)
+        row = [a, b]
+        if g == hhc.EXACT_GW:
+            row.append(_basis(kind, dims, T, tile, 1.0, 0.0, g, window=1.0) - a)
+        if all(math.isfinite(x) and x >= 0 for x in row) and t > 0 and a > 0:
+            rows.append([x / t for x in row])
+    if len(rows) < 3:
         return None
-    saa = sum(a * a for a, _ in rows); sbb = sum(b * b for _, b in rows); sab = sum(a * b for a, b in rows)
-    sa = sum(a for a, _ in rows); sb = sum(b for _, b in rows)
-    det = saa * sbb - sab * sab
-    c, tau = ((sa * sbb - sb * sab) / det, (sb * saa - sa * sab) / det) if det > 0 else (sa / saa, 0.0)
-    if tau < 0:
-        c, tau = sa / saa, 0.0
-    if c < 0:
-        c, tau = 0.0, sb / sbb
-    err = math.sqrt(sum((c * a + tau * b - 1.0) ** 2 for a, b in rows) / len(rows))
-    return {"C_iter_s": c, "tau_level_s": tau, "rel_rmse": err, "n": len(rows)}
+    x, err = _lsq(rows)
+    out = {"C_iter_s": float(x[0]), "tau_level_s": float(x[1]), "rel_rmse": err, "n": len(rows)}
+    if g == hhc.EXACT_GW:
+        out["window_rows"] = float(x[2] / x[0]) if x[0] > 0 else 0.0
+    return out
 
 
 def near_space(nd, kind, dims, T):
@@ -387,12 +425,7 @@ def sweep(args):
             continue
         best_t = min(best_t, te)
         p = {"tile": list(tile), "threads": threads, "texec": te}
-        for geom, name in ((hhc.PAPER, "talg_paper"), (hhc.EXACT, "talg_exact"), (hhc.EXACT_G, "talg_exactg")):
-            p[name] = hhc.model_predict(kind, dims, T, tile, b200_hw(cal, kind, geom, threads, tile=tile))
-        if (cal.get("exact_leff") or {}).get(str(kind)):
-            p["talg_exact_leff"] = hhc.model_predict(kind, dims, T, tile,
-                                                     b200_hw(cal, kind, hhc.EXACT, threads, leff=True,
-                                                             tile=tile))
+        predict_point(p, kind, dims, T, cal)
         pts.append(p)
         print(json.dumps(p), flush=True)
         if len(pts) % 200 == 0:            # partial results survive a killed job
@@ -400,20 +433,37 @@ def sweep(args):
     summarise_sweep(args, kind, dims, T, cal, pts, h, d_in, d_out, final=True)
 
 
+PREDICTORS = (("talg_paper", hhc.PAPER, False), ("talg_exact", hhc.EXACT, False), ("talg_exactg", hhc.EXACT_G, False),
+              ("talg_exactgw", hhc.EXACT_GW, False), ("talg_exact_leff", hhc.EXACT, True))
+
+
+def predict_point(p, kind, dims, T, cal):
+    """Talg of every predictor for a swept point (tile, threads) with calibration `cal`."""
+    tile, threads = tuple(p["tile"]), p["threads"]
+    for name, geom, lf in PREDICTORS:
+        if lf and not (cal.get("exact_leff") or {}).get(str(kind)):
+            continue
+        if geom == hhc.EXACT_GW and not (cal.get("exactgw_fit") or {}).get(str(kind)):
+            continue
+        p[name] = hhc.model_predict(kind, dims, T, tile, b200_hw(cal, kind, geom, threads, leff=lf, tile=tile))
+
+
 def summarise_sweep(args, kind, dims, T, cal, pts, h, d_in, d_out, final=True):
     """RMSE per predictor over all points and the near-best subset (reading Q15);
     with final=True also the chosen-tile gaps of the model argmins (reading Q17)."""
     best = min(pts, key=lambda p: p["texec"])
     res = {"config": args.config, "n_points": len(pts), "best_measured": best, "points": pts}
-    for name in ("talg_paper", "talg_exact", "talg_exactg", "talg_exact_leff"):
+    for name in ("talg_paper", "talg_exact", "talg_exactg", "talg_exactgw", "talg_exact_leff"):
         if not all(name in p for p in pts):
             continue
         ra, rn, nn = stats(pts, name)
         res[name] = {"rmse_all": ra, "rmse_within_20pct": rn, "n_within_20pct": nn}
     # chosen-tile gaps (reading Q17), model argmin over the swept points and over Eq. 31's space
     for geom, name, lf in (() if not final else ((hhc.PAPER, "paper", False), (hhc.EXACT, "exact", False), (hhc.EXACT_G, "exactg", False),
-                           (hhc.EXACT, "exact_leff", True))):
+                           (hhc.EXACT_GW, "exactgw", False), (hhc.EXACT, "exact_leff", True))):
         if lf and not (cal.get("exact_leff") or {}).get(str(kind)):
+            continue
+        if geom == hhc.EXACT_GW and not (cal.get("exactgw_fit") or {}).get(str(kind)):
             continue
         hw = b200_hw(cal, kind, geom, leff=lf)
         try:
@@ -453,6 +503,9 @@ def finish(args):
             if key not in seen:              # a tile measured twice keeps its first sweep's time
                 seen.add(key)
                 pts.append(p)
+    if getattr(args, "repredict", False):
+        for p in pts:
+            predict_point(p, kind, dims, T, cal)
     h = d_in = d_out = None
     if args.measure:
         a = field(CONFIG_SEEDS[args.config], dims)
@@ -460,6 +513,24 @@ def finish(args):
         d_out = torch.empty_like(d_in)
         h = hhc.stencil_create(kind, dims)
     summarise_sweep(args, kind, dims, T, cal, pts, h, d_in, d_out, final=args.measure)
+
+
+def refit(args):
+    """Refit the EXACT / EXACT_G / EXACT_GW constants (reading Q14, M10) and EXACT-Leff
+    (Q14b) from the calibration instances recorded in --cal (no kernel runs; the
+    registers of Eq. 11 are read from the device when there is one)."""
+    cal = load_cal(args.cal)
+    for key, geom in (("exact_fit", hhc.EXACT), ("exactg_fit", hhc.EXACT_G), ("exactgw_fit", hhc.EXACT_GW)):
+        cal[key] = {k: fit_exact(int(k), [(tuple(d), T_, tuple(t), v) for d, T_, t, v in inst], geom)
+                    for k, inst in cal["instances"].items()}
+    cal["exact_leff"] = {k: fit_leff(cal, int(k), [(tuple(d), T_, tuple(t), v) for d, T_, t, v in f])
+                         for k, f in (cal.get("instances_full") or {}).items()}
+    cal["fit_note"] = ("compute-only times recovered as v x the micro-benchmark's EXACT count (no register "
+                       "bound); EXACT_GW = reading M10")
+    out = args.out or args.cal
+    with open(out, "w") as f:
+        json.dump(cal, f, indent=1)
+    print(json.dumps({k: cal[k] for k in ("exact_fit", "exactg_fit", "exactgw_fit", "exact_leff")}))
 
 
 def select(args):
@@ -471,7 +542,8 @@ def select(args):
     cfg = bench.CONFIGS[args.config]
     kind, dims, T = cfg["kind"], cfg["dims"], cfg["T"]
     cal = load_cal(args.cal)
-    hw = b200_hw(cal, kind, {"paper": hhc.PAPER, "exact": hhc.EXACT, "exactg": hhc.EXACT_G}[args.geometry])
+    hw = b200_hw(cal, kind, {"paper": hhc.PAPER, "exact": hhc.EXACT, "exactg": hhc.EXACT_G,
+                             "exactgw": hhc.EXACT_GW}[args.geometry])
     t0 = time.time()
     best, thr, cands = hhc.model_select_tile(kind, dims, T, hw, args.within)
     t_sel = time.time() - t0
@@ -524,7 +596,10 @@ def main(argv=None):
     e.add_argument("--reps", type=int, default=5)
     e.add_argument("--max-measure", type=int, default=100000)
     e.add_argument("--budget", type=float, default=1800.0)
-    e.add_argument("--geometry", default="exact", choices=["paper", "exact", "exactg"])
+    e.add_argument("--geometry", default="exact", choices=["paper", "exact", "exactg", "exactgw"])
+    rf = sub.add_parser("refit")
+    rf.add_argument("--cal", default=os.path.join(ROOT, "profiles", "hw_params_b200.json"))
+    rf.add_argument("--out", default=None)
     f = sub.add_parser("finish")
     f.add_argument("--config", default="C2")
     f.add_argument("--cal", default=None)
@@ -532,8 +607,9 @@ def main(argv=None):
     f.add_argument("--out", default=None)
     f.add_argument("--reps", type=int, default=5)
     f.add_argument("--measure", action="store_true", help="time the model argmins on the GPU")
+    f.add_argument("--repredict", action="store_true", help="recompute every predictor with --cal first")
     args = ap.parse_args(argv)
-    {"calibrate": calibrate, "sweep": sweep, "select": select, "finish": finish}[args.cmd](args)
+    {"calibrate": calibrate, "sweep": sweep, "select": select, "finish": finish, "refit": refit}[args.cmd](args)
 
 
 if __name__ == "__main__":

@@ -89,9 +89,12 @@ def hw_pair(kind, geometry, rnd=None, b200=False):
         o.C_iter *= rnd.uniform(0.2, 5)
         o.tau_sync *= rnd.uniform(0.2, 5)
         o.regs_per_thread = rnd.choice([0, 0, 40, 64])
+        if geometry == hhc.EXACT_GW:
+            o.window_rows = rnd.choice([0.0, 0.3, 1.0, 2.5])
     c = hhc.make_hw(n_sm=o.nSM, n_v=o.nV, mtb_sm=o.MTBSM, r_sm=o.RSM, m_sm_bytes=o.MSM,
                     m_block_bytes=o.Mblock, L_s_per_word=o.L, tau_sync_s=o.tau_sync, T_sync_s=o.T_sync,
-                    C_iter_s=o.C_iter, regs_per_thread=o.regs_per_thread, geometry=geometry)
+                    C_iter_s=o.C_iter, regs_per_thread=o.regs_per_thread, geometry=geometry,
+                    window_rows=o.window_rows)
     return o, c
 
 
@@ -102,7 +105,7 @@ def test_model_predict_matches_oracle_hand_example(lib):
     assert abs(t - 15.96397) < 2e-5
 
 
-@pytest.mark.parametrize("geometry", [hhc.PAPER, hhc.EXACT, hhc.EXACT_G])
+@pytest.mark.parametrize("geometry", [hhc.PAPER, hhc.EXACT, hhc.EXACT_G, hhc.EXACT_GW])
 def test_model_predict_matches_oracle_random(lib, geometry):
     rnd = random.Random(geometry + 7)
     n = 0
@@ -138,7 +141,7 @@ def test_model_predict_multi_gpu_matches_oracle(lib, overlap):
     for _ in range(200):
         kind = rnd.choice([1, 2, 3, 4, 5])
         nd = hhc.KIND_NDIMS[kind]
-        geometry = rnd.choice([hhc.PAPER, hhc.EXACT, hhc.EXACT_G])
+        geometry = rnd.choice([hhc.PAPER, hhc.EXACT, hhc.EXACT_G, hhc.EXACT_GW])
         o, c = hw_pair(kind, geometry, rnd, b200=True)
         G = rnd.randint(2, 8)
         o.n_gpus = c.n_gpus = G

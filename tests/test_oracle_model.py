@@ -327,3 +327,38 @@ def test_radius_r_paper_model_hand_example():
     assert math.isclose(t, 1.6682814816e-4, rel_tol=1e-11), t
     # R = 1 is the printed model
     assert mo.talg(1, (4096,), 64, (8, 64, 0, 0), hw, R=1) == mo.talg(1, (4096,), 64, (8, 64, 0, 0), hw)
+
+
+def test_m10_window_rows_term():
+    """Reading M10 (EXACT_GW): the x-groups' window-prologue rows.  With
+    window_rows = 0 it is EXACT_G (reading M9); with L = tau = T_sync = 0 and
+    k = 1 Talg is affine in window_rows (equal steps), and by hand the slope of a
+    one-hexagon-row problem is C_iter * G * inner / nV per level per sub-tile:
+    Heat-2D S = (20, 512), T = 4, tile (4, 2, 256) with 64 threads (G = 2)."""
+    from dataclasses import replace
+    hw = mo.gtx980(2, mo.EXACT_G)
+    hw.nSM, hw.MSM, hw.Mblock = 148, 228 * 1024, 227 * 1024
+    hw.L = hw.tau_sync = hw.T_sync = 0.0
+    hw.threads = 64
+    S, T, tile = (20, 512), 4, (4, 2, 256, 0)
+    g0 = mo.talg(2, S, T, tile, hw)
+    gw = [mo.talg(2, S, T, tile, replace(hw, geometry=mo.EXACT_GW, window_rows=w)) for w in (0.0, 1.0, 2.0)]
+    assert gw[0] == g0
+    assert abs((gw[2] - gw[1]) - (gw[1] - gw[0])) <= 1e-12 * gw[2]
+    # by hand: row m has nlev levels and Nsub = ceil((S2 + nlev - 1) / tS2) sub-tiles per
+    # prism, run k at a time in ceil(ceil(w / k) / nSM) rounds (Eq. 2, 16 with m' = 0):
+    # slope = C_iter * G * tS2 / nV * sum_m nlev_m * Nsub_m * k * rounds_m
+    G, nV = 64 // (256 // 8), hw.nV
+    assert G == 2
+    slope_hand = 0.0
+    for m, lo, hi, t0 in mo.rows_exact(T, tile[0]):
+        nlev = hi - lo
+        w = mo.w_rows_exact(S[0], tile[1], tile[0])[0 if m % 2 == 0 else 1]
+        if nlev <= 0 or w == 0:
+            continue
+        nsub = mo.ceil_div(S[1] + nlev - 1, tile[2])
+        k = mo.k_exact(mo.smem_bytes_exact(2, tile), 64, hw)
+        rounds = mo.ceil_div(mo.ceil_div(w, k), hw.nSM)
+        per = nlev * nsub * rounds * (k if k > 1 else 1)
+        slope_hand += hw.C_iter * G * tile[2] / nV * per
+    assert abs((gw[1] - gw[0]) - slope_hand) <= 1e-9 * slope_hand, (gw[1] - gw[0], slope_hand)
