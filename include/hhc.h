@@ -212,7 +212,8 @@ int stencil_dist_get_unique_id(unsigned char id[128]);
 /* ncclCommInitRank on `device` (made current).  *comm receives an opaque
  * communicator owned by the library (free with stencil_dist_destroy); it also
  * owns the ghost-extended planes, the edge buffers and a second stream.
- * world = 1 needs no id and no NCCL. */
+ * world = 1 needs no id and no NCCL (with an id it still initialises a one-rank
+ * NCCL communicator: the single-GPU test of the NCCL entry points). */
 int stencil_dist_init(const unsigned char id[128], int rank, int world, int device, void** comm);
 
 /* 0 (default): exchange, then the whole ghost-extended slab per tile (2g

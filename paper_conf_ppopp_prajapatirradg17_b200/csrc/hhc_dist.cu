@@ -305,7 +305,9 @@ extern "C" int stencil_dist_init(const unsigned char id[128], int rank, int worl
     if (cudaSetDevice(device) != cudaSuccess) return STENCIL_ENODEV;
     stencil_comm_s* c = new stencil_comm_s();
     c->rank = rank; c->world = world; c->device = device;
-    if (world > 1) {
+    // NCCL for world > 1; at world 1 only when an id is given (the single-GPU test of
+    // the dlopen'ed NCCL entry points: unique id, communicator init and destroy)
+    if (world > 1 || id) {
         if (!id || !nccl().ok) { delete c; return STENCIL_ENCCL; }
         ncclUniqueId u;
         memcpy(&u, id, sizeof(u));

@@ -225,6 +225,25 @@ def test_planes_2d_pipelined_blocks(kind, dims, T, tile, threads):
         hhc.stencil_destroy(s)
 
 
+def test_dist_world1_with_nccl_communicator():
+    """The dlopen'ed NCCL entry points on one GPU: ncclGetUniqueId, a one-rank
+    ncclCommInitRank and ncclCommDestroy through stencil_dist_*, with a slab run in
+    between (world 1: no exchange) -- bit-exact against the oracle."""
+    dims, T, tile = (66, 70, 40), 9, (4, 2, 3, 32)
+    a = field(6, dims)
+    uid = hhc.stencil_dist_get_unique_id()
+    assert len(bytes(uid)) == 128
+    comm = hhc.stencil_dist_init(uid, 0, 1, 0)
+    s = hhc.stencil_create(hhc.HEAT3D_7PT, dims)
+    d_in = torch.from_numpy(a).to(DEV)
+    d_out = torch.empty_like(d_in)
+    hhc.stencil_run_dist(s, comm, d_in, d_out, T, tile)
+    torch.cuda.synchronize()
+    hhc.stencil_destroy(s)
+    hhc.stencil_dist_destroy(comm)
+    assert_bits(d_out.cpu().numpy(), oracle.run(hhc.HEAT3D_7PT, a, T, hhc.FUSED), "world 1 with NCCL")
+
+
 def test_dist_world1_nccl_free():
     """stencil_run_dist on a world-1 communicator (no NCCL needed): the slab is
     the whole grid."""
