@@ -276,6 +276,43 @@ def test_leff_fit_recovers_L(lib):
     assert abs(fit["L_s_per_word"] / Lstar - 1) < 1e-3 and fit["rel_rmse"] < 1e-3 and fit["n"] == len(full)
 
 
+@pytest.mark.parametrize("geometry", [hhc.EXACT, hhc.EXACT_G, hhc.EXACT_GW])
+def test_exact_fit_recovers_planted_constants(lib, geometry):
+    """tune.fit_exact (reading Q14; M10 for EXACT_GW): compute-only times generated
+    by the model of `geometry` with planted C_iter, tau (and window_rows), recorded
+    the way the calibration records them (as C_iter samples v = T / the
+    micro-benchmark's own EXACT count), are fitted back to the planted constants."""
+    from paper_conf_ppopp_prajapatirradg17_b200 import tune
+    kind = hhc.HEAT2D_9PT if geometry != hhc.EXACT_GW else hhc.HEAT3D_7PT
+    C, tau, w = 1.3e-8, 2.2e-8, 0.7
+    rnd = random.Random(11 + geometry)
+    insts = []
+    while len(insts) < 40:
+        if kind == hhc.HEAT2D_9PT:
+            dims = (rnd.randint(1024, 4096), rnd.randint(1024, 4096))
+            tile = (2 * rnd.randint(1, 16), rnd.randint(1, 32), 32 * rnd.randint(1, 16), 0)
+            T = rnd.randint(16, 64)
+        else:
+            dims = (rnd.randint(96, 256), rnd.randint(96, 256), rnd.randint(96, 256))
+            tile = (2 * rnd.randint(1, 6), rnd.randint(1, 8), rnd.randint(1, 6), 32 * rnd.randint(1, 2))
+            T = rnd.randint(8, 24)
+        hw = tune.b200_hw(None, kind, geometry)
+        hw.C_iter_s, hw.tau_sync_s, hw.L_s_per_word, hw.T_sync_s = C, tau, 0.0, 0.0
+        hw.window_rows = w if geometry == hhc.EXACT_GW else 0.0
+        t = hhc.model_predict(kind, dims, T, tile, hw)
+        cnt = tune._micro_count(kind, dims, T, tile)
+        if math.isfinite(t) and math.isfinite(cnt) and cnt > 0:
+            insts.append((dims, T, tile, t / cnt))
+    fit = tune.fit_exact(kind, insts, geometry)
+    # the model is linear in (C_iter, tau, C_iter * window_rows) up to Eq. 16's max(m', c) on
+    # time-clipped rows (m' = 2 tau when L = 0): near-exact, not exact
+    tol = 1e-2 if kind == hhc.HEAT2D_9PT else 5e-2           # 3D: more rows where m' > c
+    assert fit["rel_rmse"] < tol and fit["n"] == len(insts), fit
+    assert abs(fit["C_iter_s"] / C - 1) < tol and abs(fit["tau_level_s"] / tau - 1) < 2 * tol, fit
+    if geometry == hhc.EXACT_GW:
+        assert abs(fit["window_rows"] / w - 1) < 4 * tol, fit
+
+
 @pytest.mark.parametrize("geometry", [hhc.PAPER, hhc.EXACT])
 def test_model_radius_r_matches_oracle(lib, geometry):
     """f4 kinds (radius R = 2..4, reading F4): C++ model_predict vs the oracle,
