@@ -969,6 +969,7 @@ extern "C" int stencil_hexdist_connect(stencil_t h, void* hd, const unsigned cha
         for (int i = 0; i < 3; ++i)
             if (cudaIpcOpenMemHandle(&ptr[i], hh[i], cudaIpcMemLazyEnablePeerAccess) != cudaSuccess) {
                 cudaGetLastError();
+                for (int j = 0; j < i; ++j) cudaIpcCloseMemHandle(ptr[j]);   // no half-open neighbour
                 return STENCIL_ECUDA;
             }
         int64_t part[6];
