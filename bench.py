@@ -43,7 +43,7 @@ CONFIGS = {
     "C4": dict(kind=4, dims=(512, 512, 512), T=256, tile=(8, 8, 16, 64), threads=512,
                tiles_by_gpus={2: (8, 6, 16, 64), 4: (8, 2, 16, 64), 8: (6, 2, 16, 64)},
                desc="Heat-3D 7-point fp32, 512^3, T=256"),
-    "C5": dict(kind=5, dims=(768, 768, 768), T=128, tile=(8, 6, 8, 64), threads=256,
+    "C5": dict(kind=5, dims=(768, 768, 768), T=128, tile=(8, 10, 14, 64), threads=448,
                tiles_by_gpus={8: (8, 2, 16, 64)}, threads_by_gpus={8: 512},
                desc="Laplacian-3D 27-point fp32, 768^3, T=128"),
     # SURVEY §8(f) f2 (not a BASELINE.json config): the paper's 1D derivation case
