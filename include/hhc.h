@@ -139,6 +139,15 @@ int stencil_run(stencil_t h, const float* d_in, float* d_out, int64_t T,
 int stencil_run_host(stencil_t h, const float* h_in, float* h_out, int64_t T,
                      stencil_tile tile, int threads, void* cuda_stream);
 
+/* n independent problems (same handle, T and tile) from/to HOST buffers h_in[i] ->
+ * h_out[i] (n_elements floats each; pinned for overlap), pipelined: the
+ * host-to-device copy of problem i+1 and the device-to-host copy of problem i-1
+ * run on the library's own copy streams while problem i runs on cuda_stream
+ * (two device buffer pairs, allocated at first use, owned by the handle).
+ * Results as n calls of stencil_run_host.  Synchronises. */
+int stencil_run_host_batch(stencil_t h, int n, const float* const* h_in, float* const* h_out, int64_t T,
+                           stencil_tile tile, int threads, void* cuda_stream);
+
 /* Predicted execution time Talg in seconds (Eqs. 2-30).
  * dims are full ABI extents (the model uses S = dims-2).  Returns NaN for
  * invalid arguments and +INFINITY for an infeasible tile (Eq. 31 constraints),

@@ -100,6 +100,8 @@ def load(build_if_missing: bool = False):
     lib.stencil_destroy.restype = None
     lib.stencil_run.argtypes = [vp, vp, vp, ctypes.c_int64, stencil_tile, ctypes.c_int, vp]
     lib.stencil_run_host.argtypes = [vp, vp, vp, ctypes.c_int64, stencil_tile, ctypes.c_int, vp]
+    lib.stencil_run_host_batch.argtypes = [vp, ctypes.c_int, ctypes.POINTER(vp), ctypes.POINTER(vp), ctypes.c_int64,
+                                           stencil_tile, ctypes.c_int, vp]
     lib.stencil_run_planes.argtypes = [vp, ctypes.c_int64, vp, vp, ctypes.c_int64, stencil_tile,
                                        ctypes.c_int, vp]
     lib.model_predict.argtypes = [ctypes.c_int, ctypes.c_int, i64p, ctypes.c_int64, stencil_tile,
@@ -231,6 +233,17 @@ def stencil_run(s: Stencil, d_in, d_out, T: int, tile, threads: int = 0, stream=
 def stencil_run_host(s: Stencil, h_in, h_out, T: int, tile, threads: int = 0, stream=None):
     _check(load().stencil_run_host(s.handle, _ptr(h_in), _ptr(h_out), int(T), make_tile(tile), int(threads),
                                    _stream(stream)), "stencil_run_host")
+
+
+def stencil_run_host_batch(s: Stencil, h_ins, h_outs, T: int, tile, threads: int = 0, stream=None):
+    """n problems host -> device -> host with the copies overlapping the runs (the C call)."""
+    n = len(h_ins)
+    if n != len(h_outs) or n < 1:
+        raise ValueError("stencil_run_host_batch: h_ins and h_outs must have the same non-zero length")
+    ins = (ctypes.c_void_p * n)(*[_ptr(x) for x in h_ins])
+    outs = (ctypes.c_void_p * n)(*[_ptr(x) for x in h_outs])
+    _check(load().stencil_run_host_batch(s.handle, n, ins, outs, int(T), make_tile(tile), int(threads),
+                                         _stream(stream)), "stencil_run_host_batch")
 
 
 def stencil_run_planes(s: Stencil, rows: int, plane0, plane1, T: int, tile, threads: int = 0, stream=None):
@@ -420,7 +433,7 @@ def updates(dims, T: int, kind: int = 0) -> int:
     return int(T) * math.prod(int(x) - 2 * R for x in dims)
 
 
-EXPORTED_SYMBOLS = ["stencil_create", "stencil_destroy", "stencil_run", "stencil_run_host",
+EXPORTED_SYMBOLS = ["stencil_create", "stencil_destroy", "stencil_run", "stencil_run_host", "stencil_run_host_batch",
                     "stencil_run_planes", "model_predict", "model_select_tile", "stencil_tile_resources", "stencil_tile_occupancy",
                     "stencil_plan_info", "stencil_microbench", "stencil_strerror", "stencil_last_launches",
                     "stencil_profile", "stencil_run_wavefront", "stencil_wavefront_info",

@@ -89,6 +89,9 @@ struct stencil_s {
     int64_t faceg_n = 0;
     float* h_in_dev = nullptr;   // stencil_run_host device buffers
     float* h_out_dev = nullptr;
+    float* hb_dev[2][2] = {{nullptr, nullptr}, {nullptr, nullptr}};   // stencil_run_host_batch [slot][in/out]
+    cudaStream_t hb_s[2] = {nullptr, nullptr};                       // its copy streams (H2D, D2H)
+    cudaEvent_t hb_ev[2][3] = {{nullptr, nullptr, nullptr}, {nullptr, nullptr, nullptr}};
     int sticky = 0;
     int64_t last_launches = 0;
     cudaStream_t cap_stream = nullptr;
@@ -211,6 +214,13 @@ extern "C" void stencil_destroy(stencil_t h) {
     if (h->faceg) cudaFree(h->faceg);
     if (h->h_in_dev) cudaFree(h->h_in_dev);
     if (h->h_out_dev) cudaFree(h->h_out_dev);
+    for (int i = 0; i < 2; ++i) {
+        for (int j = 0; j < 2; ++j)
+            if (h->hb_dev[i][j]) cudaFree(h->hb_dev[i][j]);
+        if (h->hb_s[i]) cudaStreamDestroy(h->hb_s[i]);
+        for (int j = 0; j < 3; ++j)
+            if (h->hb_ev[i][j]) cudaEventDestroy(h->hb_ev[i][j]);
+    }
     if (h->cap_stream) cudaStreamDestroy(h->cap_stream);
     delete h;
 }
@@ -609,6 +619,60 @@ extern "C" int stencil_run_host(stencil_t h, const float* h_in, float* h_out, in
     e = cudaMemcpyAsync(h_out, h->h_out_dev, n * sizeof(float), cudaMemcpyDeviceToHost, s);
     if (e != cudaSuccess) return cuda_fail(h, e);
     return cuda_fail(h, cudaStreamSynchronize(s));
+}
+
+// n independent problems from/to host buffers, pipelined over two device buffer
+// pairs: the H2D copy of problem i+1 (own stream) and the D2H copy of problem i-1
+// (own stream) overlap the HHC rows of problem i on cuda_stream.  Events order
+// every buffer reuse: in[k] is refilled after the run that read it, out[k] is
+// rewritten after its D2H.  Synchronises before returning.
+extern "C" int stencil_run_host_batch(stencil_t h, int n, const float* const* h_in, float* const* h_out, int64_t T,
+                                      stencil_tile tile, int threads, void* cuda_stream) {
+    if (!h || n < 1 || !h_in || !h_out) return STENCIL_EINVAL;
+    if (h->sticky) return h->sticky;
+    for (int i = 0; i < n; ++i)
+        if (!h_in[i] || !h_out[i]) return STENCIL_EINVAL;
+    const int64_t n_el = h->nelem();
+    const size_t bytes = (size_t)n_el * sizeof(float);
+    cudaStream_t s = (cudaStream_t)cuda_stream;
+    cudaSetDevice(h->device);
+    if (!h->hb_dev[0][0]) {
+        for (int k = 0; k < 2; ++k) {
+            for (int j = 0; j < 2; ++j)
+                if (cudaMalloc(&h->hb_dev[k][j], bytes) != cudaSuccess) { h->hb_dev[k][j] = nullptr; return STENCIL_ENOMEM; }
+            if (cudaStreamCreateWithFlags(&h->hb_s[k], cudaStreamNonBlocking) != cudaSuccess) return STENCIL_ECUDA;
+            for (int j = 0; j < 3; ++j)
+                if (cudaEventCreateWithFlags(&h->hb_ev[k][j], cudaEventDisableTiming) != cudaSuccess) return STENCIL_ECUDA;
+        }
+    }
+    cudaStream_t sin = h->hb_s[0], sout = h->hb_s[1];
+    // per slot k: ev[k][0] = input copied, ev[k][1] = run done, ev[k][2] = output copied
+    cudaError_t e = cudaSuccess;
+    auto upload = [&](int i) {
+        const int k = i & 1;
+        if (i >= 2) cudaStreamWaitEvent(sin, h->hb_ev[k][1], 0);       // the run of i-2 read in[k]
+        e = cudaMemcpyAsync(h->hb_dev[k][0], h_in[i], bytes, cudaMemcpyHostToDevice, sin);
+        cudaEventRecord(h->hb_ev[k][0], sin);
+    };
+    cudaEventRecord(h->hb_ev[1][1], s);        // orders the first uploads after earlier work on s
+    cudaStreamWaitEvent(sin, h->hb_ev[1][1], 0);
+    upload(0);
+    for (int i = 0; i < n && e == cudaSuccess; ++i) {
+        const int k = i & 1;
+        if (i + 1 < n) upload(i + 1);
+        cudaStreamWaitEvent(s, h->hb_ev[k][0], 0);                     // input i on the device
+        if (i >= 2) cudaStreamWaitEvent(s, h->hb_ev[k][2], 0);         // out[k] copied out (problem i-2)
+        int rc = stencil_run(h, h->hb_dev[k][0], h->hb_dev[k][1], T, tile, threads, cuda_stream);
+        if (rc) return rc;
+        cudaEventRecord(h->hb_ev[k][1], s);
+        cudaStreamWaitEvent(sout, h->hb_ev[k][1], 0);
+        e = cudaMemcpyAsync(h_out[i], h->hb_dev[k][1], bytes, cudaMemcpyDeviceToHost, sout);
+        cudaEventRecord(h->hb_ev[k][2], sout);
+    }
+    if (e != cudaSuccess) return cuda_fail(h, e);
+    e = cudaStreamSynchronize(sout);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+    return cuda_fail(h, e);
 }
 
 // ---- wavefront-parallel Jacobi-1D (reading W1)

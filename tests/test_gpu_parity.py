@@ -225,6 +225,22 @@ def test_planes_2d_pipelined_blocks(kind, dims, T, tile, threads):
         hhc.stencil_destroy(s)
 
 
+def test_run_host_batch_pipelined():
+    """stencil_run_host_batch: independent problems from/to pinned host buffers
+    with the copies overlapping the runs (two device buffer pairs); every result
+    equals the oracle, 2D and 3D, n = 1..5 (buffer reuse after two steps)."""
+    for kind, dims, T, tile in ((hhc.HEAT2D_9PT, (70, 130), 17, (6, 3, 32)),
+                                (hhc.HEAT3D_7PT, (20, 22, 40), 7, (4, 2, 3, 32))):
+        s = hhc.stencil_create(kind, dims)
+        for n in (1, 2, 5):
+            ins = [torch.from_numpy(field(700 + 10 * n + i, dims)).pin_memory() for i in range(n)]
+            outs = [torch.empty(dims, dtype=torch.float32).pin_memory() for _ in range(n)]
+            hhc.stencil_run_host_batch(s, ins, outs, T, tile)
+            for i in range(n):
+                assert_bits(outs[i].numpy(), oracle.run(kind, ins[i].numpy(), T, hhc.FUSED), f"batch n={n} i={i}")
+        hhc.stencil_destroy(s)
+
+
 def test_dist_world1_with_nccl_communicator():
     """The dlopen'ed NCCL entry points on one GPU: ncclGetUniqueId, a one-rank
     ncclCommInitRank and ncclCommDestroy through stencil_dist_*, with a slab run in
