@@ -38,7 +38,8 @@ CONFIGS = {
     # tiles_by_gpus: the tile per GPU count under torchrun, the best measured on one GPU for
     # the slab each rank holds (scripts/slab_tiles.py -> profiles/r02/slab_C{3,4,5}.json)
     "C3": dict(kind=3, dims=(16384, 16384), T=512, tile=(32, 12, 512, 0), threads=384,
-               tiles_by_gpus={2: (32, 12, 512, 0), 4: (24, 4, 512, 0), 8: (16, 4, 512, 0)},
+               tiles_by_gpus={2: (32, 12, 512, 0), 4: (24, 3, 512, 0), 8: (12, 3, 512, 0)},
+               threads_by_gpus={4: 512, 8: 512},
                desc="Gradient-2D fp32, 16384x16384, T=512"),
     "C4": dict(kind=4, dims=(512, 512, 512), T=256, tile=(8, 8, 16, 64), threads=512,
                tiles_by_gpus={2: (8, 6, 16, 64), 4: (8, 2, 16, 64), 8: (6, 2, 16, 64)},

@@ -30,8 +30,11 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
 
 
-def candidates(nd, rows):
-    if nd == 2:
+def candidates(nd, rows, wide=False):
+    if nd == 2 and wide:
+        out = [((tT, tS1, tS2, 0), thr) for tT in (4, 6, 8, 10, 12, 16, 20, 24) for tS1 in (2, 3, 4, 6, 8)
+               for tS2 in (256, 512) for thr in ((tS2 // 8) * g for g in (2, 3, 4, 6, 8)) if thr <= 512]
+    elif nd == 2:
         out = [((tT, tS1, tS2, 0), thr) for tT in (8, 16, 24, 32) for tS1 in (4, 8, 12, 16) for tS2 in (256, 512)
                for thr in ((tS2 // 8) * g for g in (2, 3, 6)) if thr <= 384]
     else:
@@ -54,6 +57,7 @@ def main():
     ap.add_argument("--reps", type=int, default=3)
     ap.add_argument("--budget", type=float, default=900.0)
     ap.add_argument("--out", default=None)
+    ap.add_argument("--wide", action="store_true", help="2D: a denser candidate set (small hexagons, up to 512 threads)")
     args = ap.parse_args()
     cfg = bench.CONFIGS[args.config]
     kind, dims, T = cfg["kind"], cfg["dims"], cfg["T"]
@@ -89,7 +93,7 @@ def main():
             hhc.stencil_destroy(h)
             return (n - 1) * tt[tT] + tt[Tl]
 
-        for tile, thr in candidates(nd, own + 2 * 32):
+        for tile, thr in candidates(nd, own + 2 * 32, args.wide):
             if time.time() - t_start > args.budget:
                 break
             try:
