@@ -62,3 +62,25 @@ def test_torchrun_hexdist_path_world1():
               "--master-port", "29534", "bench.py", "--gpus", "2", "--config", "C1", "--exchange", "hexdist",
               "--steps", "2", "--warmup", "3"])
     assert d["n_gpus"] == 1 and d["value"] > 0 and "f1" in d["config"]["parallelism"]
+
+
+def test_bench_launch_configs_are_valid_tiles():
+    """Every launch configuration bench.py can time -- the config tile/threads and
+    the per-GPU-count tiles under torchrun -- passes the library's tile validation
+    (host-only planner rules: smem, threads per kind, integrality)."""
+    sys.path.insert(0, ROOT)
+    import bench
+    import paper_conf_ppopp_prajapatirradg17_b200 as hhc
+    from paper_conf_ppopp_prajapatirradg17_b200 import dist
+    for name, c in bench.CONFIGS.items():
+        nd = len(c["dims"])
+        tiles = {1: (tuple(c["tile"]), c["threads"])}
+        for n in (2, 4, 8):
+            t, thr, _ = dist.choose_tile(c, n) if nd > 1 else (tuple(c["tile"]), c["threads"], 0)
+            tiles[n] = (t, thr)
+        for n, (t, thr) in tiles.items():
+            t = tuple(t) + (0,) * (4 - len(t))
+            if c.get("schedule") == "wavefront":
+                continue
+            smem, block, _ = hhc.stencil_tile_resources(nd, t, thr, kind=c["kind"])
+            assert block == thr and smem <= 227 * 1024, (name, n, t, thr)
